@@ -1,0 +1,161 @@
+"""Invariants that pin the oracle GA (P@21534-22160).
+
+The GA trajectory itself has no reference in the paper ("parity unpinned",
+DESIGN.md §3); what the paper and the mathematics fix are checked here:
+elitism keeps the best, children respect the block-count range, the search
+reaches the exhaustive optimum on small chains (Fig. 5's "optimal within 15
+generations", P@35749-35945), and never beats the exact DP optimum.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+
+SEEDS = [1, 42, 20230807]
+
+
+def _popcount_rows(pop, n):
+    W = pop.shape[-1]
+    c = np.zeros(pop.shape[:-1], dtype=np.int64)
+    for w in range(W):
+        x = pop[..., w].copy()
+        if w == W - 1 and (n - 1) % 64:
+            x &= np.uint64((1 << ((n - 1) % 64)) - 1)
+        c += np.array([bin(int(v)).count("1") for v in x.reshape(-1)]).reshape(x.shape)
+    return c
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("ovh_kind", ["profile", "const", "zero", "ties"])
+def test_c1_fixed_k_ga_finds_brute_force_optimum(seed, ovh_kind):
+    """C1 as the paper runs it — one GA per fixed block count (Table 3, Fig. 5 'RES-1 =
+    2 blocks', P@35254-35716): each reaches the exhaustive optimum (bits included)."""
+    lat, ovh = wl.c1_chain(overhead=ovh_kind)
+    for k in range(2, 13):
+        b = oracle.brute(lat, ovh, k, k)
+        r = oracle.ga_run(lat, ovh, 50, seed, pop_size=256, n_elite=4, k_min=k, k_max=k)
+        assert r["fitness"] == b["fitness"] and int(r["bits"][0]) == b["bits"], k
+        assert r["generations_run"] == 50
+        assert r["evaluations"] == 256 + 50 * 252
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+def test_c1_range_mode_near_optimum(seed):
+    """Range mode k in [2, 12] is multimodal in k: the GA never beats brute force and its
+    best is within the top 1% of the 2047 splits."""
+    lat, ovh = wl.c1_chain()
+    b = oracle.brute(lat, ovh, 2, 12)
+    r = oracle.ga_run(lat, ovh, 50, seed, pop_size=256, n_elite=4, k_min=2, k_max=12)
+    allf = sorted((oracle.fitness(lat, ovh, np.array([m], np.uint64), 2, 12)["fitness"]
+                   for m in range(1, 2048)), reverse=True)
+    assert r["fitness"] <= b["fitness"]
+    assert allf.index(r["fitness"]) < 21
+
+
+def test_c1_tie_chain_canonical():
+    lat, ovh = wl.c1_chain(overhead="ties")
+    b = oracle.brute(lat, ovh, 2, 12)
+    r = oracle.ga_run(lat, ovh, 50, 7, pop_size=256, n_elite=4, k_min=2, k_max=12)
+    assert r["fitness"] == b["fitness"] and int(r["bits"][0]) == b["bits"]
+
+
+def test_elitism_monotone_and_k_range():
+    lat, ovh = wl.chain("resnet50_122")
+    n = len(lat)
+    prev = -math.inf
+    prev_f = None
+    for g in range(0, 12):
+        r = oracle.ga_run(lat, ovh, g, 5, pop_size=128, n_elite=4, k_min=3, k_max=9, want_population=True)
+        f = r["fitness_all"][0]
+        fmax = f.max()
+        assert fmax >= prev
+        prev = fmax
+        assert r["fitness"] >= fmax          # record covers the current population
+        k = _popcount_rows(r["population"], n) + 1
+        assert k.min() >= 3 and k.max() <= 9
+        # elites: slots 0..E-1 hold the E best of the previous generation, in rank order
+        if prev_f is not None:
+            assert np.array_equal(f[:4], np.sort(prev_f)[::-1][:4])
+        prev_f = f
+
+
+def test_full_elite_freezes_population():
+    lat, ovh = wl.chain("vgg16")
+    r0 = oracle.ga_run(lat, ovh, 0, 3, pop_size=64, n_elite=64, k_min=2, k_max=8, want_population=True)
+    r5 = oracle.ga_run(lat, ovh, 5, 3, pop_size=64, n_elite=64, k_min=2, k_max=8, want_population=True)
+    rows0 = sorted(map(tuple, r0["population"][0].tolist()))
+    rows5 = sorted(map(tuple, r5["population"][0].tolist()))
+    assert rows0 == rows5
+    assert np.all(np.diff(r5["fitness_all"][0]) <= 0)
+
+
+def test_no_variation_children_are_parents():
+    lat, ovh = wl.chain("mobilenetv2")
+    n = len(lat)
+    kw = dict(pop_size=100, n_elite=2, k_min=1, k_max=n, p_crossover=0.0, p_mutation=0.0, want_population=True)
+    r0 = oracle.ga_run(lat, ovh, 0, 11, **kw)
+    r1 = oracle.ga_run(lat, ovh, 1, 11, **kw)
+    parents = set(map(tuple, r0["population"][0].tolist()))
+    assert set(map(tuple, r1["population"][0].tolist())) <= parents
+
+
+def test_init_respects_front_skip_and_k():
+    lat, ovh = wl.chain("bert_base")
+    n = len(lat)
+    r = oracle.ga_run(lat, ovh, 0, 9, pop_size=512, n_elite=8, k_min=4, k_max=4, front_skip=200,
+                      want_population=True)
+    pop = r["population"][0]
+    assert np.all(_popcount_rows(pop, n) == 3)
+    assert np.all(pop[:, :3] == 0)                          # positions < 192 untouched
+    assert np.all(pop[:, 3] & np.uint64((1 << 8) - 1) == 0)  # positions 192..199
+
+
+@pytest.mark.parametrize("k", [2, 3, 4])
+def test_ga_never_beats_dp_and_reaches_it(k):
+    # fixed-k runs on a paper-shaped chain with constant overhead: the DP optimum bounds
+    # the GA, and the search should reach it quickly (Fig. 5, P@35749-35945)
+    lat, _ = wl.chain("vgg16")
+    ovh, delta = wl.constant_overhead(lat)
+    n = len(lat)
+    v = oracle.dp(lat, delta, k)
+    f_dp = oracle.fitness_from(k, int(v[k]), (k - 1) * delta, int(lat.sum()))
+    r = oracle.ga_run(lat, ovh, 30, 1, pop_size=256, n_elite=4, k_min=k, k_max=k)
+    assert r["fitness"] <= f_dp
+    assert r["fitness"] == f_dp
+    assert r["var_num"] == v[k]
+
+
+def test_stall_termination():
+    lat, ovh = wl.c1_chain()
+    r = oracle.ga_run(lat, ovh, 500, 1, pop_size=256, n_elite=4, k_min=2, k_max=12, stall_generations=15)
+    assert r["generations_run"] < 500
+    assert r["generations_run"] - r["generation_found"] >= 15 or r["generation_found"] == 0
+
+
+def test_islands_deterministic_and_migration_invariants():
+    lat, ovh = wl.chain("resnet50_175")
+    kw = dict(pop_size=128, n_elite=4, k_min=2, k_max=16, n_islands=4, migration_interval=3, n_migrants=4)
+    a = oracle.ga_run(lat, ovh, 9, 77, want_population=True, **kw)
+    b = oracle.ga_run(lat, ovh, 9, 77, want_population=True, **kw)
+    assert np.array_equal(a["population"], b["population"])
+    assert a["evaluations"] == 4 * (128 + 9 * 124)
+    # the global record is the best over all islands' final populations at least
+    assert a["fitness"] >= a["fitness_all"].max()
+    # with migration the islands share individuals; without, island 0 runs alone
+    solo = oracle.ga_run(lat, ovh, 9, 77, pop_size=128, n_elite=4, k_min=2, k_max=16, want_population=True)
+    nomig = oracle.ga_run(lat, ovh, 9, 77, want_population=True, **{**kw, "migration_interval": 0})
+    assert np.array_equal(nomig["population"][0], solo["population"][0])
+    assert not np.array_equal(a["population"][0], solo["population"][0])
+
+
+def test_invalid_params_rejected():
+    lat, ovh = wl.c1_chain()
+    with pytest.raises(ValueError):
+        oracle.ga_run(lat, ovh, 1, 1, pop_size=255, n_elite=4)     # (N - E) odd
+    with pytest.raises(ValueError):
+        oracle.ga_run(lat, ovh, 1, 1, pop_size=256, n_elite=4, tournament_size=33)
+    with pytest.raises(ValueError):
+        oracle.ga_run(lat, ovh, 1, 1, pop_size=256, n_elite=4, k_min=5, k_max=4)
