@@ -1,0 +1,363 @@
+#!/usr/bin/env python
+"""Benchmark of the GA split search (SPLIT, ICPP'23 §3.3) on B200.
+
+Metric (BASELINE.json): split-candidate fitness evals/sec and GA generations/sec.
+
+A step = one split_ga_run(): generation 0 (init + eval of N candidates) and
+500 generations of elite top-E, tournament, crossover, mutation, repair and
+fused fitness evaluation, on the C2 workload (BASELINE.json configs[1]:
+ResNet-50-shaped chain of 175 ops, population 65,536 per island).  With
+--gpus N (torchrun, one rank per GPU) every rank runs one island of that size
+(weak scaling) and islands exchange their top-64 over NCCL every 10
+generations.  Rank 0 prints one JSON line.
+
+--impl reference times the CPU oracle (oracle/, plain C, one thread) on a
+bounded sample of the same workload — the only other place bench.py runs it.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "split-candidate fitness evals/sec and GA generations/sec at 1/2/4/8 B200"
+UNIT = "evals/s"
+C2 = dict(chain="resnet50_175", pop_size=65536, n_elite=1024, tournament_size=4, p_crossover=0.9,
+          p_mutation=0.2, k_min=2, k_max=32, generations=500)
+MIGRATION_INTERVAL, N_MIGRANTS = 10, 64
+C5_EVAL_N = 1 << 24           # split_eval_batch sub-measurement (C5: n = 1024, 2.3 GB of bitsets > L2)
+CPU_SAMPLE_GENERATIONS = 100  # oracle cpu_baseline: about 10 s of one core
+REF_STEP_GENERATIONS = 10     # --impl reference: oracle generations per step
+
+
+def _workload_desc(world: int) -> dict:
+    return {
+        "workload": "C2 (BASELINE configs[1]): ResNet-50-shaped chain n=175 ops (W=3 words, T=28.35 ms, "
+                    "profile-style cut overheads), GA pop=65536 per island, E=1024, s=4, pc=0.9, pm=0.2, "
+                    "k in [2,32], 500 generations per step",
+        "islands": world, "pop_per_island": C2["pop_size"], "generations_per_step": C2["generations"],
+        "migration": (f"top-{N_MIGRANTS} every {MIGRATION_INTERVAL} generations over NCCL" if world > 1 else "none"),
+        "l2": "flushed between timed steps (256 MiB write); the 1.7 MB population itself is L2-resident",
+        "parallelism": f"island-dp{world}",
+    }
+
+
+def _peaks() -> dict:
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "src": "fallback"}
+
+
+def _profile_traffic(name: str):
+    """dram bytes per launch from the committed ncu summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get(name)
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100",
+                 "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.lines = []
+        if self.proc:
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [ln for ln in out.splitlines() if ln.strip()]
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in getattr(self, "lines", []):
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def _dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def ga_bytes_per_generation(N: int, E: int, W: int, s: int) -> int:
+    """Algorithmic HBM bytes of one generation: per child one parent row
+    read (pairs read two rows for two children), one child row and one f64 written, s
+    f64 tournament gathers; the elite step reads N f64 and copies E rows + f64."""
+    return (N - E) * (16 * W + 8 + 8 * s) + 8 * N + 2 * E * (8 * W + 8)
+
+
+def eval_bytes_per_candidate(W: int) -> int:
+    return 8 * W + 8
+
+
+def cpu_baseline_oracle(generations: int) -> dict:
+    import oracle
+    from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+    lat, ovh = wl.chain(C2["chain"])
+    kw = {k: C2[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max")}
+    t0 = time.perf_counter()
+    r = oracle.ga_run(lat, ovh, generations, 1, **kw)
+    dt = time.perf_counter() - t0
+    return {"value": r["evaluations"] / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"oracle GA (plain C, 1 thread) on C2: N=65536, {generations} generations "
+                      f"({r['evaluations']} evals) in {dt:.2f} s",
+            "gens_per_s": generations / dt}
+
+
+def run_reference(args):
+    world, rank, _ = _dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+    lat, ovh = wl.chain(C2["chain"])
+    kw = {k: C2[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max")}
+    G = REF_STEP_GENERATIONS
+    for i in range(args.warmup):
+        oracle.ga_run(lat, ovh, 1, 100 + i, **kw)
+    evals, t0 = 0, time.perf_counter()
+    for i in range(args.steps):
+        evals += oracle.ga_run(lat, ovh, G, i, **kw)["evaluations"]
+    dt = time.perf_counter() - t0
+    value = evals / dt
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1000 / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64/f64",
+        "data": "synthetic", "config": {**_workload_desc(1), "reference_sample": f"{G} generations per step"},
+        "gens_per_s": args.steps * G / dt,
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"oracle GA on C2, N=65536, {G} generations per step x {args.steps} steps"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--generations", type=int, default=C2["generations"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-eval", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icpp_luoyww0023_b200 import split as S
+    from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+
+    world, rank, local = _dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    comm = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        uid = [S.split_comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = S.split_comm_init(uid[0], rank, world, local)
+    stream = torch.cuda.current_stream()
+    lat, ovh = wl.chain(C2["chain"])
+    G = args.generations
+    gkw = {k: C2[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max")}
+    isl = dict(island_id=rank, n_islands=world, islands_per_device=1,
+               migration_interval=MIGRATION_INTERVAL if world > 1 else 0, n_migrants=N_MIGRANTS if world > 1 else 0)
+    h = S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl)
+    W = h.W
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+
+    for i in range(args.warmup):
+        h.run(G, 1000 + i)
+    torch.cuda.synchronize()
+
+    step_ms, evals, launches, loop_ms, gens, n_general, n_fast = [], 0, 0, [], 0, 0, 0
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    best = None
+    with ClockSampler(local) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        wall0 = time.perf_counter()
+        for i in range(args.steps):
+            flush.fill_(i & 0xFF)                    # L2 flush between timed steps (not timed)
+            ev0[i].record(stream)
+            r = h.run(G, i)
+            ev1[i].record(stream)
+            st = h.last_run_stats()
+            evals += r["evaluations"]
+            gens += r["generations_run"]
+            launches += st["launches"]
+            loop_ms.append(st["ms_loop"])
+            n_general += st["general_selects"]
+            n_fast += st["fast_selects"]
+            best = r
+        torch.cuda.synchronize()
+        barrier()
+        wall = time.perf_counter() - wall0
+    for i in range(args.steps):
+        step_ms.append(ev0[i].elapsed_time(ev1[i]))
+    t_ms = sum(step_ms)
+    t = torch.tensor([t_ms, wall * 1000.0], dtype=torch.float64, device=dev)
+    tot = torch.tensor([float(evals), float(gens)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+    t_max_ms, wall_max_ms = float(t[0]), float(t[1])
+    evals_all = float(tot[0])
+    value = evals_all / (t_max_ms / 1000.0)
+    gens_per_s = (gens / (t_max_ms / 1000.0))           # generations of the GA (island-parallel)
+
+    # roofline of the dominant kernel: the persistent GA kernel's generation loop
+    peaks = _peaks()
+    gen_bytes = ga_bytes_per_generation(C2["pop_size"], C2["n_elite"], W, C2["tournament_size"])
+    loop_avg_ms = sum(loop_ms) / len(loop_ms)
+    achieved_gbs = gen_bytes * G / (loop_avg_ms / 1000.0) / 1e9
+    roofline = {"bound": "hbm", "kernel": "ga_kernel (RUN segment: all generations of a step)",
+                "achieved": achieved_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved_gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
+                "traffic": _profile_traffic("ga_kernel_per_generation"),
+                "algorithmic_bytes_per_generation": gen_bytes,
+                "launch_ms_avg": loop_avg_ms, "share_of_step": loop_avg_ms / (t_max_ms / args.steps)}
+
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_max_ms / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int64/f64", "data": "synthetic",
+        "config": _workload_desc(world), "gens_per_s": gens_per_s,
+        "wall_ms_per_step": wall_max_ms / args.steps, "gpu_launches": launches,
+        "elite_select_paths": {"radix_general": n_general, "candidate_merge": n_fast},
+        "best": {"fitness": best["fitness"], "k": best["k"], "generation_found": best["generation_found"]},
+        "roofline": roofline,
+    }
+
+    # split_eval_batch at C5 (HBM-bound; the north-star's >= 60 % target)
+    if not args.no_eval:
+        lat5, ovh5 = wl.chain("synthetic_1024")
+        h5 = S.SplitGA(lat5, ovh5, pop_size=4, n_elite=0, k_min=2, k_max=32, device=local, stream=stream)
+        W5 = h5.W
+        bits = torch.from_numpy(wl.uniform_k_population_fast(len(lat5), C5_EVAL_N, seed=20230807).view(np.int64)).to(dev)
+        fout = torch.empty(C5_EVAL_N, dtype=torch.float64, device=dev)
+        for _ in range(3):
+            h5.eval_batch(bits, C5_EVAL_N, fout)
+        torch.cuda.synchronize()
+        e0 = [torch.cuda.Event(enable_timing=True) for _ in range(10)]
+        e1 = [torch.cuda.Event(enable_timing=True) for _ in range(10)]
+        for i in range(10):
+            flush.fill_(i)
+            e0[i].record(stream)
+            h5.eval_batch(bits, C5_EVAL_N, fout)
+            e1[i].record(stream)
+        torch.cuda.synchronize()
+        ms = [a.elapsed_time(b) for a, b in zip(e0, e1)]
+        ms_avg = sum(ms) / len(ms)
+        bpc = eval_bytes_per_candidate(W5)
+        gbs = bpc * C5_EVAL_N / (ms_avg / 1000.0) / 1e9
+        out["eval_batch"] = {
+            "workload": "C5: synthetic 1024-op chain (W=16), N=2^24 candidates, k ~ U[2,32]",
+            "evals_per_s": C5_EVAL_N / (ms_avg / 1000.0), "ms_per_launch": ms_avg,
+            "roofline": {"bound": "hbm", "kernel": "eval_batch_kernel", "achieved": gbs, "peak": peaks["hbm_gbs"],
+                         "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
+                         "traffic": _profile_traffic("eval_batch_kernel_c5"),
+                         "algorithmic_bytes_per_candidate": bpc}}
+        h5.close()
+        del bits, fout
+
+    # e2e through the public API with host buffers: create (H2D of the chain) + run + best (D2H)
+    if not args.no_e2e:
+        e2e_steps = max(3, min(args.steps, 10))
+        e_evals = 0
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for i in range(e2e_steps):
+            with S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl) as he:
+                e_evals += he.run(G, 5000 + i)["evaluations"]
+        torch.cuda.synchronize()
+        barrier()
+        et = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        ee = torch.tensor([float(e_evals)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+            dist.all_reduce(ee, op=dist.ReduceOp.SUM)
+        n = len(lat)
+        h2d = 4 * (((n + 1 + 3) & ~3) + ((n - 1 + 3) & ~3)) + 8   # staged chain words + best bits
+        d2h = 48 + world * (W + 2) * 8 + 5 * 8 + 8                # control block, island records, best stats
+        out["e2e"] = {"value": float(ee[0]) / float(et[0]), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                      "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+                      "note": "split_ga_create(host latencies) + split_ga_run + best to host + destroy, wall clock"}
+
+    out["clocks"] = clk.summary()
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline_oracle(CPU_SAMPLE_GENERATIONS)
+    out["paper_context"] = ("PAPER.md profiles 'over 20,000 candidates' offline on a Jetson Nano at ~1 s per "
+                            "candidate (287,980 candidates > 80 h, P@9901-10019): ~1 eval/s; context only")
+    h.close()
+    if comm:
+        S.split_comm_destroy(comm)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,186 @@
+/*
+ * split_ga.h — C ABI of the B200 GA split search (SPLIT, ICPP'23, §3.3).
+ *
+ * The library searches for "evenly-sized" splits of a model's operator chain:
+ * m-1 cut points divide the model into m blocks (PAPER.md P@20780-20831) and a
+ * genetic algorithm maximises Eq. 2 (P@21101-21296)
+ *
+ *     fitness = -( e^(sigma/T - 1) + e^(overhead/m - 1) )
+ *
+ * where sigma is the (population) standard deviation of the block execution
+ * times, T the vanilla model's execution time and overhead the splitting
+ * overhead ratio (fn. 2, P@13393-13520).  The GA steps follow P@21534-22160;
+ * every detail the paper leaves open is fixed by the readings R1-R19 of
+ * DESIGN.md §3.  Algorithm 1 (greedy preemption, P@27209-28515) is exposed as
+ * a host-only decision function.
+ *
+ * Conventions
+ *  - Every entry point returns an int status: SPLIT_OK (0) or a negative
+ *    SPLIT_E_* code; split_strerror() names it and split_last_error() gives a
+ *    thread-local detail string.  Nothing is thrown across the ABI.
+ *  - Device work runs on the handle's stream (params.stream, a cudaStream_t;
+ *    NULL = the legacy default stream) and device params.device.
+ *  - Bitset layout: candidate c is row c of a dense row-major uint64_t[N][W],
+ *    W = ceil((n_ops-1)/64) words (split_words()).  Bit p of the row (word
+ *    p>>6, bit p&63) means "cut between operator p and operator p+1",
+ *    p in [0, n_ops-2].  Bits >= n_ops-1 in the last word are padding: ignored.
+ *  - Integer-ns latencies; block times, S1 = sum t, S2 = sum t^2 and
+ *    V = k*S2 - S1^2 (= k^2 sigma^2) are exact integers; the FP64 tail
+ *    follows DESIGN.md R5'/R5'' so results are bit-reproducible.
+ *  - A handle is not thread-safe; distinct handles are independent.
+ */
+#ifndef SPLIT_GA_H
+#define SPLIT_GA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+    SPLIT_OK = 0,
+    SPLIT_E_INVAL = -1,  /* null pointer, zero size, out-of-range parameter   */
+    SPLIT_E_RANGE = -2,  /* latency/overhead magnitudes break the int guards  */
+    SPLIT_E_ALIGN = -3,  /* device buffer not 16-byte (bits) / 8-byte aligned */
+    SPLIT_E_NOMEM = -4,  /* device or host allocation failed                  */
+    SPLIT_E_CUDA = -5,   /* CUDA runtime error (see split_last_error)         */
+    SPLIT_E_NCCL = -6,   /* NCCL error or NCCL not loadable                   */
+    SPLIT_E_STATE = -7   /* call not valid in the handle's state              */
+};
+
+typedef struct split_ga_t split_ga_t;  /* opaque; owns device state */
+
+/* GA parameters.  Paper-silent choices and their defaults: DESIGN.md R6-R11,
+ * R16-R18.  split_ga_params_default() fills every field. */
+typedef struct {
+    uint32_t pop_size;          /* N individuals per island, >= 2                        */
+    uint32_t n_elite;           /* E, 0..min(N,1024); (N - E) must be even  (P@21965-22054) */
+    uint32_t tournament_size;   /* s, 1..32                                  (R7)        */
+    double p_crossover;         /* [0,1]  one-point crossover probability    (P@21745-21902) */
+    double p_mutation;          /* [0,1]  per-child one-bit-flip probability (P@21906-21963) */
+    uint32_t k_min, k_max;      /* block-count range, 1 <= k_min <= k_max <= n_ops (R6)  */
+    uint32_t front_skip;        /* init draws cut positions from [front_skip, n_ops-2]
+                                   (observation "far from the front", P@19343-19437)     */
+    uint32_t stall_generations; /* stop after this many generations without a strictly
+                                   better fitness; 0 = off               (P@22056-22160) */
+    const int64_t* cut_overhead_ns; /* host, n_ops-1 entries: extra time the block after
+                                   cut p pays (R3); NULL = all 0.  Copied at create.     */
+    uint32_t island_id;         /* first global island this handle runs                 */
+    uint32_t n_islands;         /* total islands across all ranks                       */
+    uint32_t islands_per_device;/* islands this handle runs: [island_id, +islands_per_device) */
+    uint32_t migration_interval;/* M: migrate every M generations (0 = off)     (R16)   */
+    uint32_t n_migrants;        /* K: migrants per island, 1 <= K <= N - E when M > 0    */
+    void* comm;                 /* split_comm_init() communicator when islands span ranks,
+                                   NULL when every island is on this device              */
+    int device;                 /* CUDA device ordinal                                   */
+    void* stream;               /* cudaStream_t for all device work (NULL = default)     */
+} split_ga_params;
+
+void split_ga_params_default(split_ga_params* p);
+
+/* a0 — validate and stage a chain.  latencies_ns: host, n_ops >= 2 entries,
+ * each >= 0, sum T >= 1.  Computes the exclusive prefix P[0..n], copies
+ * P and the overheads to the device (u32), sets the Bernoulli thresholds and
+ * allocates the population for islands_per_device islands.
+ * Guards (SPLIT_E_RANGE): T' = T + (sum of the k_max-1 largest overheads) must
+ * be < 2^32 and (k_max-1)*T'^2 < 2^63 so every segment sum fits u32, S2 fits
+ * u64 and V fits int64.  *out is set only on success. */
+int split_ga_create(const int64_t* latencies_ns, uint32_t n_ops, const split_ga_params* p,
+                    split_ga_t** out);
+
+uint32_t split_words(const split_ga_t* h);  /* W = ceil((n_ops-1)/64); 0 on NULL */
+
+/* a2 — score candidates with Eq. 2.  cut_bitsets: DEVICE pointer to n_cand*W
+ * words, 16-byte aligned (SPLIT_E_ALIGN); fitness_out: DEVICE pointer to n_cand
+ * doubles, 8-byte aligned.  Candidates with k outside [k_min, k_max] get
+ * -INFINITY.  Asynchronous on the handle's stream; buffers are caller-owned and
+ * must live until the stream work completes.  n_cand = 0 is a no-op. */
+int split_eval_batch(split_ga_t* h, const uint64_t* cut_bitsets, uint64_t n_cand, double* fitness_out);
+
+/* a2 through HOST buffers: copies the bitsets in, evaluates and copies the
+ * fitness back in chunks, overlapping copies with compute.  Synchronous.  Any
+ * host pointers are accepted; page-locked ones are fastest. */
+int split_eval_batch_host(split_ga_t* h, const uint64_t* cut_bitsets_host, uint64_t n_cand,
+                          double* fitness_out_host);
+
+/* Best split found.  bits: caller-owned HOST buffer of split_words() words. */
+typedef struct {
+    uint64_t* bits;
+    double fitness;
+    uint32_t k;                 /* number of blocks m                          */
+    int64_t var_num;            /* V = k*S2 - S1^2 = k^2 sigma^2               */
+    uint64_t s1, s2;            /* sum t_j, sum t_j^2 (ns, ns^2)               */
+    uint64_t overhead_ns;       /* sum of the cut overheads                    */
+    double expected_wait_ns;    /* Eq. 1: S2 / (2 S1)   (P@17226-17827)        */
+    uint32_t generation_found;  /* generation the record was first reached     */
+    uint32_t generations_run;   /* transitions performed (< generations on stall) */
+    uint64_t evaluations;       /* fitness evaluations by this handle          */
+} split_best_t;
+
+/* a1, a3-a9 — run the GA: init generation 0 from seed (re-initialises on every
+ * call), then up to `generations` transitions (R11).  With islands across
+ * ranks every rank must call it with the same arguments; best_out then holds
+ * the GLOBAL best on every rank.  Synchronous. */
+int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, split_best_t* best_out);
+
+/* Copy the current population of local island `local_island` (after the last
+ * split_ga_run) to host buffers bits_host[N*W] and fitness_host[N] (either may
+ * be NULL).  For tests and checkpointing.  Synchronous. */
+int split_ga_population(split_ga_t* h, uint32_t local_island, uint64_t* bits_host, double* fitness_host);
+
+/* a10 — Algorithm 1 greedy preemption (host only, O(n)).  queue[0] is the head
+ * (runs next), queue[n-1] the tail.  *insert_pos receives the index at which
+ * the incoming request is inserted (0 = head, n = behind the tail).
+ * SPLIT_E_INVAL when ext_ns <= 0, ext_left_ns not in [0, ext_ns] (any request),
+ * alpha <= 0, queue == NULL with n > 0, or insert_pos == NULL.
+ * Under reading R12 the decision reduces to: scanning from the tail, pass t_i
+ * iff its type differs and ext_left(t_i)*ext(t_i) > ext_left(new)*ext(new). */
+typedef struct {
+    uint32_t type_id;
+    int64_t arrival_ns, ext_ns, ext_left_ns;
+} split_request;
+typedef struct {
+    int64_t now_ns;
+    double alpha;               /* latency target = alpha * Ext (fn. 3, P@29746-29870) */
+    uint32_t n;
+    const split_request* queue; /* host, n entries, [0] = head */
+    split_request incoming;
+} split_queue_state;
+int split_preempt_decide(const split_queue_state* q, uint32_t* insert_pos);
+
+/* Island communicator over NCCL (the libnccl.so.2 already loaded in the
+ * process, e.g. by torch).  Rank r of `world` runs islands_per_device islands
+ * starting at island_id = r*islands_per_device.  unique_id: 128 bytes from
+ * rank 0, broadcast by the caller (e.g. torch.distributed).  Collective. */
+int split_comm_unique_id(uint8_t out[128]);
+int split_comm_init(const uint8_t id[128], int rank, int world, int device, void** comm);
+void split_comm_destroy(void* comm);
+
+void split_ga_destroy(split_ga_t* h);
+const char* split_strerror(int code);
+const char* split_last_error(void);
+
+/* Diagnostics (device self-tests used by the parity tests): evaluate the
+ * device Philox4x32-10 on n (ctr[4], key[2]) tuples and the device dexp on n
+ * doubles.  Host buffers; synchronous.  device = CUDA ordinal. */
+int split_selftest_philox(int device, const uint32_t* ctr_key /* n*6 */, uint32_t n, uint32_t* out /* n*4 */);
+int split_selftest_dexp(int device, const double* z, uint32_t n, double* out);
+
+/* Timing support for bench.py: number of kernel launches the last
+ * split_ga_run / split_eval_batch issued, and the device time (ms, CUDA events
+ * on the handle's stream) of the last split_ga_run's generation loop and of its
+ * dominant kernel. */
+typedef struct {
+    uint64_t launches;
+    float ms_total;
+    float ms_loop;
+    uint32_t general_selects;   /* generations that needed the radix top-E path */
+    uint32_t fast_selects;      /* generations served by the candidate merge     */
+} split_run_stats;
+int split_last_run_stats(const split_ga_t* h, split_run_stats* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPLIT_GA_H */

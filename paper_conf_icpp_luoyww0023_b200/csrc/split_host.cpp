@@ -1,0 +1,732 @@
+// split_host.cpp — C ABI of include/split_ga.h: validation, chain staging (a0),
+// the GA driver around the persistent kernel (segments, sync points, island
+// migration over NCCL), best-record assembly, Algorithm 1 (a10, host only).
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <math.h>
+#include <nccl.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+#include <vector>
+
+#include "split_ga.h"
+#include "split_internal.h"
+
+using namespace splitga;
+
+// ------------------------------------------------------------------------
+// errors
+// ------------------------------------------------------------------------
+static thread_local char g_err[512];
+
+static int fail(int code, const char* fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return code;
+}
+
+#define CU(call)                                                                                  \
+    do {                                                                                          \
+        cudaError_t e_ = (call);                                                                  \
+        if (e_ != cudaSuccess)                                                                    \
+            return fail(SPLIT_E_CUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+extern "C" const char* split_last_error(void) { return g_err; }
+
+extern "C" const char* split_strerror(int code)
+{
+    switch (code) {
+    case SPLIT_OK: return "ok";
+    case SPLIT_E_INVAL: return "invalid argument";
+    case SPLIT_E_RANGE: return "latency/overhead magnitudes exceed the exact-integer guards";
+    case SPLIT_E_ALIGN: return "misaligned device buffer";
+    case SPLIT_E_NOMEM: return "out of memory";
+    case SPLIT_E_CUDA: return "CUDA error";
+    case SPLIT_E_NCCL: return "NCCL error";
+    case SPLIT_E_STATE: return "invalid state";
+    default: return "unknown error";
+    }
+}
+
+// ------------------------------------------------------------------------
+// NCCL, resolved at run time from the libnccl.so.2 already in the process
+// (torch's), so the library never pins a second NCCL build.
+// ------------------------------------------------------------------------
+struct NcclApi {
+    ncclResult_t (*getUniqueId)(ncclUniqueId*);
+    ncclResult_t (*commInitRank)(ncclComm_t*, int, ncclUniqueId, int);
+    ncclResult_t (*allGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t);
+    ncclResult_t (*commDestroy)(ncclComm_t);
+    const char* (*getErrorString)(ncclResult_t);
+    bool ok;
+};
+
+static NcclApi* nccl_api()
+{
+    static NcclApi api{};
+    static bool tried = false;
+    if (tried) return api.ok ? &api : nullptr;
+    tried = true;
+    void* h = nullptr;
+    const char* env = getenv("SPLIT_NCCL_LIB");
+    if (env && *env) h = dlopen(env, RTLD_NOW | RTLD_LOCAL);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_LOCAL);
+    if (!h) return nullptr;
+    api.getUniqueId = (decltype(api.getUniqueId))dlsym(h, "ncclGetUniqueId");
+    api.commInitRank = (decltype(api.commInitRank))dlsym(h, "ncclCommInitRank");
+    api.allGather = (decltype(api.allGather))dlsym(h, "ncclAllGather");
+    api.commDestroy = (decltype(api.commDestroy))dlsym(h, "ncclCommDestroy");
+    api.getErrorString = (decltype(api.getErrorString))dlsym(h, "ncclGetErrorString");
+    api.ok = api.getUniqueId && api.commInitRank && api.allGather && api.commDestroy && api.getErrorString;
+    return api.ok ? &api : nullptr;
+}
+
+struct SplitComm {
+    ncclComm_t comm;
+    int rank, world, device;
+};
+
+extern "C" int split_comm_unique_id(uint8_t out[128])
+{
+    if (!out) return fail(SPLIT_E_INVAL, "split_comm_unique_id: out is NULL");
+    NcclApi* api = nccl_api();
+    if (!api) return fail(SPLIT_E_NCCL, "libnccl.so.2 not loadable (set SPLIT_NCCL_LIB)");
+    ncclUniqueId id;
+    ncclResult_t r = api->getUniqueId(&id);
+    if (r != ncclSuccess) return fail(SPLIT_E_NCCL, "ncclGetUniqueId: %s", api->getErrorString(r));
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    memcpy(out, &id, 128);
+    return SPLIT_OK;
+}
+
+extern "C" int split_comm_init(const uint8_t id[128], int rank, int world, int device, void** comm)
+{
+    if (!id || !comm || world < 1 || rank < 0 || rank >= world) return fail(SPLIT_E_INVAL, "split_comm_init: bad args");
+    NcclApi* api = nccl_api();
+    if (!api) return fail(SPLIT_E_NCCL, "libnccl.so.2 not loadable (set SPLIT_NCCL_LIB)");
+    CU(cudaSetDevice(device));
+    ncclUniqueId uid;
+    memcpy(&uid, id, 128);
+    SplitComm* c = new (std::nothrow) SplitComm{};
+    if (!c) return fail(SPLIT_E_NOMEM, "split_comm_init: host alloc");
+    ncclResult_t r = api->commInitRank(&c->comm, world, uid, rank);
+    if (r != ncclSuccess) {
+        delete c;
+        return fail(SPLIT_E_NCCL, "ncclCommInitRank: %s", api->getErrorString(r));
+    }
+    c->rank = rank;
+    c->world = world;
+    c->device = device;
+    *comm = c;
+    return SPLIT_OK;
+}
+
+extern "C" void split_comm_destroy(void* comm)
+{
+    if (!comm) return;
+    SplitComm* c = (SplitComm*)comm;
+    NcclApi* api = nccl_api();
+    if (api) api->commDestroy(c->comm);
+    delete c;
+}
+
+// ------------------------------------------------------------------------
+// handle
+// ------------------------------------------------------------------------
+struct split_ga_t {
+    split_ga_params p;
+    uint32_t n, W;
+    uint64_t T;
+    int device;
+    cudaStream_t stream;
+    int num_sms;
+    ChainDev ch;
+    GaArgs ga;
+    int grid;
+    uint32_t cpi;
+    std::vector<void*> allocs;
+    // host-side state
+    uint32_t last_gen;
+    bool have_pop;
+    split_run_stats stats;
+    // scratch
+    int64_t* d_stats;
+    double* d_statf;
+    uint64_t* d_bits1;
+    uint64_t* d_recpack;   // [I_total][W + 2]
+    cudaEvent_t ev[4];
+    // eval_batch_host staging
+    uint64_t* d_hbits[2];
+    double* d_hfit[2];
+    uint64_t h_chunk;
+    cudaStream_t hs[2];
+};
+
+extern "C" void split_ga_params_default(split_ga_params* p)
+{
+    if (!p) return;
+    memset(p, 0, sizeof(*p));
+    p->pop_size = 65536;
+    p->n_elite = 1024;
+    p->tournament_size = 4;
+    p->p_crossover = 0.9;
+    p->p_mutation = 0.2;
+    p->k_min = 2;
+    p->k_max = 32;
+    p->front_skip = 0;
+    p->stall_generations = 0;
+    p->cut_overhead_ns = nullptr;
+    p->island_id = 0;
+    p->n_islands = 1;
+    p->islands_per_device = 1;
+    p->migration_interval = 0;
+    p->n_migrants = 0;
+    p->comm = nullptr;
+    p->device = 0;
+    p->stream = nullptr;
+}
+
+extern "C" uint32_t split_words(const split_ga_t* h) { return h ? h->W : 0; }
+
+static void free_all(split_ga_t* h)
+{
+    for (void* q : h->allocs) cudaFree(q);
+    h->allocs.clear();
+    for (int i = 0; i < 4; ++i)
+        if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+    for (int i = 0; i < 2; ++i)
+        if (h->hs[i]) cudaStreamDestroy(h->hs[i]);
+}
+
+template <class T>
+static int dalloc(split_ga_t* h, T** out, size_t count)
+{
+    void* q = nullptr;
+    size_t bytes = count * sizeof(T);
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(&q, bytes);
+    if (e != cudaSuccess) return fail(SPLIT_E_NOMEM, "cudaMalloc(%zu): %s", bytes, cudaGetErrorString(e));
+    h->allocs.push_back(q);
+    e = cudaMemset(q, 0, bytes);
+    if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "cudaMemset: %s", cudaGetErrorString(e));
+    *out = (T*)q;
+    return SPLIT_OK;
+}
+
+static uint64_t bern_thr(double p)
+{
+    if (!(p > 0.0)) return 0;
+    if (p >= 1.0) return (uint64_t)1 << 32;
+    return (uint64_t)floor(p * 4294967296.0);
+}
+
+static uint32_t pow2_at_least(uint32_t x)
+{
+    uint32_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+#define TRY(x)                  \
+    do {                        \
+        int rc_ = (x);          \
+        if (rc_ != SPLIT_OK) {  \
+            free_all(h);        \
+            delete h;           \
+            return rc_;         \
+        }                       \
+    } while (0)
+
+extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_params* pp, split_ga_t** out)
+{
+    if (!lat || !pp || !out) return fail(SPLIT_E_INVAL, "split_ga_create: NULL argument");
+    const split_ga_params p = *pp;
+    if (n < 2 || n > 64u * kMaxWords + 1) return fail(SPLIT_E_INVAL, "n_ops must be in [2, %u]", 64u * kMaxWords + 1);
+    unsigned __int128 T = 0;
+    for (uint32_t i = 0; i < n; ++i) {
+        if (lat[i] < 0) return fail(SPLIT_E_INVAL, "latencies_ns[%u] < 0", i);
+        T += (uint64_t)lat[i];
+    }
+    if (T < 1) return fail(SPLIT_E_INVAL, "sum of latencies must be >= 1");
+    if (p.pop_size < 2) return fail(SPLIT_E_INVAL, "pop_size must be >= 2");
+    if (p.n_elite > p.pop_size || p.n_elite > kMaxElite) return fail(SPLIT_E_INVAL, "n_elite must be <= min(N, %u)", kMaxElite);
+    if ((p.pop_size - p.n_elite) & 1u) return fail(SPLIT_E_INVAL, "pop_size - n_elite must be even");
+    if (p.tournament_size < 1 || p.tournament_size > 32) return fail(SPLIT_E_INVAL, "tournament_size must be in [1, 32]");
+    if (!(p.p_crossover >= 0.0 && p.p_crossover <= 1.0) || !(p.p_mutation >= 0.0 && p.p_mutation <= 1.0))
+        return fail(SPLIT_E_INVAL, "probabilities must be in [0, 1]");
+    if (p.k_min < 1 || p.k_min > p.k_max || p.k_max > n) return fail(SPLIT_E_INVAL, "need 1 <= k_min <= k_max <= n_ops");
+    if (p.front_skip > n - 2 || p.k_max - 1 > n - 1 - p.front_skip)
+        return fail(SPLIT_E_INVAL, "k_max - 1 cut points do not fit in [front_skip, n_ops-2]");
+    if (p.islands_per_device < 1 || p.islands_per_device > kMaxLocalIslands)
+        return fail(SPLIT_E_INVAL, "islands_per_device must be in [1, %u]", kMaxLocalIslands);
+    if (p.n_islands < p.islands_per_device || p.island_id + p.islands_per_device > p.n_islands)
+        return fail(SPLIT_E_INVAL, "island range outside [0, n_islands)");
+    if ((uint64_t)p.n_islands * p.pop_size >= (1ull << 32)) return fail(SPLIT_E_INVAL, "n_islands * pop_size must be < 2^32");
+    if (p.n_islands > p.islands_per_device && !p.comm)
+        return fail(SPLIT_E_INVAL, "islands span ranks but comm is NULL");
+    const bool migrate = p.migration_interval > 0 && p.n_islands > 1;
+    if (migrate && (p.n_migrants < 1 || p.n_migrants > p.pop_size - p.n_elite || p.n_migrants > kMaxElite))
+        return fail(SPLIT_E_INVAL, "n_migrants must be in [1, min(N - E, %u)]", kMaxElite);
+    std::vector<int64_t> ovh(n - 1, 0);
+    if (p.cut_overhead_ns) {
+        for (uint32_t i = 0; i + 1 < n; ++i) {
+            if (p.cut_overhead_ns[i] < 0) return fail(SPLIT_E_INVAL, "cut_overhead_ns[%u] < 0", i);
+            ovh[i] = p.cut_overhead_ns[i];
+        }
+    }
+    // exact-integer guards (a0)
+    std::vector<int64_t> srt(ovh);
+    std::sort(srt.begin(), srt.end(), std::greater<int64_t>());
+    unsigned __int128 Tp = T;
+    for (uint32_t i = 0; i + 1 < p.k_max && i < srt.size(); ++i) Tp += (uint64_t)srt[i];
+    if (Tp >= ((unsigned __int128)1 << 32)) return fail(SPLIT_E_RANGE, "T + largest overheads must be < 2^32 ns");
+    if ((unsigned __int128)(p.k_max - 1) * Tp * Tp >= ((unsigned __int128)1 << 63))
+        return fail(SPLIT_E_RANGE, "(k_max-1) * T'^2 must be < 2^63");
+
+    split_ga_t* h = new (std::nothrow) split_ga_t();
+    if (!h) return fail(SPLIT_E_NOMEM, "host alloc");
+    h->p = p;
+    h->p.cut_overhead_ns = nullptr;
+    h->n = n;
+    h->W = (n - 1 + 63) / 64;
+    h->T = (uint64_t)T;
+    h->device = p.device;
+    h->stream = (cudaStream_t)p.stream;
+    {
+        cudaError_t e = cudaSetDevice(p.device);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, p.device);
+        if (e != cudaSuccess) {
+            delete h;
+            return fail(SPLIT_E_CUDA, "device %d: %s", p.device, cudaGetErrorString(e));
+        }
+    }
+    // chain words: P[0..n] padded to x4, ovh[0..n-2] padded to x4
+    const uint32_t p_words = (n + 1 + 3) & ~3u, o_words = (n - 1 + 3) & ~3u;
+    std::vector<uint32_t> words(p_words + o_words, 0);
+    uint64_t acc = 0;
+    for (uint32_t i = 0; i < n; ++i) {
+        words[i] = (uint32_t)acc;
+        acc += (uint64_t)lat[i];
+    }
+    words[n] = (uint32_t)acc;
+    for (uint32_t i = 0; i + 1 < n; ++i) words[p_words + i] = (uint32_t)ovh[i];
+    uint32_t* d_chain = nullptr;
+    TRY(dalloc(h, &d_chain, words.size()));
+    {
+        cudaError_t e = cudaMemcpy(d_chain, words.data(), words.size() * 4, cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) {
+            free_all(h);
+            delete h;
+            return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
+        }
+    }
+    ChainDev& ch = h->ch;
+    ch.words = d_chain;
+    ch.n = n;
+    ch.W = h->W;
+    ch.p_words = p_words;
+    ch.o_words = o_words;
+    ch.T = (uint32_t)acc;
+    ch.k_min = p.k_min;
+    ch.k_max = p.k_max;
+    const uint32_t rem = (n - 1) & 63u;
+    ch.last_mask = rem ? ((1ull << rem) - 1) : ~0ull;
+
+    GaArgs& a = h->ga;
+    memset(&a, 0, sizeof(a));
+    a.ch = ch;
+    a.N = p.pop_size;
+    a.E = p.n_elite;
+    a.s = p.tournament_size;
+    a.K = migrate ? p.n_migrants : 0;
+    a.I = p.islands_per_device;
+    a.island_base = p.island_id;
+    a.I_total = p.n_islands;
+    a.front_skip = p.front_skip;
+    a.stall = p.stall_generations;
+    a.thr_c = bern_thr(p.p_crossover);
+    a.thr_m = bern_thr(p.p_mutation);
+    uint32_t sc = std::max<uint32_t>(pow2_at_least(kCandCap), pow2_at_least(std::max<uint32_t>(a.E, 2)));
+    if (migrate) sc = std::max(sc, pow2_at_least((p.n_islands - 1) * a.K));
+    a.sort_cap = sc;
+    if (ga_smem_bytes(a) > 227 * 1024) {
+        free_all(h);
+        delete h;
+        return fail(SPLIT_E_INVAL, "shared-memory plan %zu B exceeds 227 KB (n_ops, islands or migrants too large)",
+                    ga_smem_bytes(a));
+    }
+    cudaError_t ge;
+    h->grid = ga_grid(a, h->num_sms, &ge);
+    if (ge != cudaSuccess || h->grid < (int)a.I) {
+        free_all(h);
+        delete h;
+        return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s", cudaGetErrorString(ge));
+    }
+    h->cpi = (uint32_t)h->grid / a.I;
+    const size_t IN = (size_t)a.I * a.N;
+    for (int b = 0; b < 2; ++b) {
+        TRY(dalloc(h, &a.pop[b], IN * h->W));
+        TRY(dalloc(h, &a.fit[b], IN));
+        TRY(dalloc(h, &a.cand_key[b], IN));
+        TRY(dalloc(h, &a.cand_idx[b], IN));
+    }
+    TRY(dalloc(h, &a.cand_cnt, 2 * (size_t)a.I));
+    TRY(dalloc(h, &a.sel_key, (size_t)a.I * kMaxElite));
+    TRY(dalloc(h, &a.sel_idx, (size_t)a.I * kMaxElite));
+    TRY(dalloc(h, &a.sel_cnt, a.I));
+    TRY(dalloc(h, &a.tau, a.I));
+    TRY(dalloc(h, &a.ghist, 3 * (size_t)a.I * 256));
+    TRY(dalloc(h, &a.part_f, 2 * (size_t)a.I * h->cpi));
+    TRY(dalloc(h, &a.part_idx, 2 * (size_t)a.I * h->cpi));
+    TRY(dalloc(h, &a.rec_f, a.I));
+    TRY(dalloc(h, &a.rec_bits, (size_t)a.I * h->W));
+    TRY(dalloc(h, &a.rec_gen, a.I));
+    TRY(dalloc(h, &a.rec_valid, a.I));
+    TRY(dalloc(h, &a.mig_bits, (size_t)a.I_total * std::max<uint32_t>(a.K, 1) * h->W));
+    TRY(dalloc(h, &a.mig_f, (size_t)a.I_total * std::max<uint32_t>(a.K, 1)));
+    TRY(dalloc(h, &a.ctl, 1));
+    TRY(dalloc(h, &h->d_stats, 8));
+    TRY(dalloc(h, &h->d_statf, 1));
+    TRY(dalloc(h, &h->d_bits1, h->W));
+    TRY(dalloc(h, &h->d_recpack, (size_t)a.I_total * (h->W + 2)));
+    for (int i = 0; i < 4; ++i) {
+        cudaError_t e = cudaEventCreate(&h->ev[i]);
+        if (e != cudaSuccess) TRY(fail(SPLIT_E_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
+    }
+    *out = h;
+    return SPLIT_OK;
+}
+
+extern "C" void split_ga_destroy(split_ga_t* h)
+{
+    if (!h) return;
+    cudaSetDevice(h->device);
+    cudaStreamSynchronize(h->stream);
+    free_all(h);
+    delete h;
+}
+
+// ------------------------------------------------------------------------
+// a2 eval
+// ------------------------------------------------------------------------
+extern "C" int split_eval_batch(split_ga_t* h, const uint64_t* bits, uint64_t n_cand, double* out)
+{
+    if (!h) return fail(SPLIT_E_INVAL, "split_eval_batch: NULL handle");
+    if (n_cand == 0) return SPLIT_OK;
+    if (!bits || !out) return fail(SPLIT_E_INVAL, "split_eval_batch: NULL buffer");
+    if (((uintptr_t)bits & 15u) || ((uintptr_t)out & 7u)) return fail(SPLIT_E_ALIGN, "bitsets must be 16-byte aligned, fitness 8-byte");
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, bits) != cudaSuccess || at.type != cudaMemoryTypeDevice) {
+        cudaGetLastError();
+        if (!(at.type == cudaMemoryTypeManaged)) return fail(SPLIT_E_INVAL, "cut_bitsets is not a device pointer");
+    }
+    CU(cudaSetDevice(h->device));
+    h->stats.launches = 0;
+    CU(launch_eval_batch(h->ch, bits, n_cand, out, h->stream, h->num_sms, &h->stats.launches));
+    return SPLIT_OK;
+}
+
+extern "C" int split_eval_batch_host(split_ga_t* h, const uint64_t* bits_host, uint64_t n_cand, double* fit_host)
+{
+    if (!h) return fail(SPLIT_E_INVAL, "split_eval_batch_host: NULL handle");
+    if (n_cand == 0) return SPLIT_OK;
+    if (!bits_host || !fit_host) return fail(SPLIT_E_INVAL, "split_eval_batch_host: NULL buffer");
+    CU(cudaSetDevice(h->device));
+    const uint64_t chunk = 1ull << 22;  // candidates per pipeline stage
+    if (h->h_chunk == 0) {
+        for (int b = 0; b < 2; ++b) {
+            int rc = dalloc(h, &h->d_hbits[b], chunk * h->W);
+            if (rc) return rc;
+            rc = dalloc(h, &h->d_hfit[b], chunk);
+            if (rc) return rc;
+            CU(cudaStreamCreateWithFlags(&h->hs[b], cudaStreamNonBlocking));
+        }
+        h->h_chunk = chunk;
+    }
+    CU(cudaStreamSynchronize(h->stream));
+    h->stats.launches = 0;
+    for (uint64_t c = 0, k = 0; c < n_cand; c += chunk, ++k) {
+        const int b = (int)(k & 1);
+        const uint64_t m = std::min<uint64_t>(chunk, n_cand - c);
+        CU(cudaMemcpyAsync(h->d_hbits[b], bits_host + c * h->W, m * h->W * 8, cudaMemcpyHostToDevice, h->hs[b]));
+        CU(launch_eval_batch(h->ch, h->d_hbits[b], m, h->d_hfit[b], h->hs[b], h->num_sms, &h->stats.launches));
+        CU(cudaMemcpyAsync(fit_host + c, h->d_hfit[b], m * 8, cudaMemcpyDeviceToHost, h->hs[b]));
+    }
+    CU(cudaStreamSynchronize(h->hs[0]));
+    CU(cudaStreamSynchronize(h->hs[1]));
+    return SPLIT_OK;
+}
+
+// ------------------------------------------------------------------------
+// a1, a3-a9: the GA driver
+// ------------------------------------------------------------------------
+static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
+{
+    GaArgs a = h->ga;
+    a.mode = mode;
+    a.g_begin = g0;
+    a.g_end = g1;
+    cudaError_t e = launch_ga(a, h->stream, h->num_sms, &h->stats.launches);
+    if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "GA kernel (mode %u): %s", mode, cudaGetErrorString(e));
+    return SPLIT_OK;
+}
+
+static bool rec_better(double fa, const uint64_t* a, double fb, const uint64_t* b, uint32_t W)
+{
+    if (fa != fb) return fa > fb;
+    for (int w = (int)W - 1; w >= 0; --w)
+        if (a[w] != b[w]) return a[w] < b[w];
+    return false;
+}
+
+// all-gather a device buffer: each rank contributes `bytes` at offset rank*bytes
+static int allgather(split_ga_t* h, void* base, size_t bytes)
+{
+    SplitComm* c = (SplitComm*)h->p.comm;
+    if (!c || c->world == 1) return SPLIT_OK;
+    NcclApi* api = nccl_api();
+    if (!api) return fail(SPLIT_E_NCCL, "NCCL not loadable");
+    const char* src = (const char*)base + (size_t)c->rank * bytes;
+    ncclResult_t r = api->allGather(src, base, bytes, ncclUint8, c->comm, h->stream);
+    if (r != ncclSuccess) return fail(SPLIT_E_NCCL, "ncclAllGather: %s", api->getErrorString(r));
+    return SPLIT_OK;
+}
+
+struct GlobalRec {
+    double f;
+    uint32_t gen;
+    std::vector<uint64_t> bits;
+};
+
+// gather island records across ranks; returns the global best (R19)
+static int global_record(split_ga_t* h, GlobalRec* best)
+{
+    const uint32_t W = h->W, I = h->ga.I, It = h->ga.I_total;
+    const size_t stride = W + 2;
+    // pack local records at this rank's slot: [f bits][gen][W words]
+    uint64_t* slot = h->d_recpack + (size_t)h->ga.island_base * stride;
+    for (uint32_t i = 0; i < I; ++i) {
+        CU(cudaMemcpyAsync(slot + i * stride, h->ga.rec_f + i, 8, cudaMemcpyDeviceToDevice, h->stream));
+        CU(cudaMemcpyAsync(slot + i * stride + 1, h->ga.rec_gen + i, 4, cudaMemcpyDeviceToDevice, h->stream));
+        CU(cudaMemcpyAsync(slot + i * stride + 2, h->ga.rec_bits + (size_t)i * W, W * 8, cudaMemcpyDeviceToDevice, h->stream));
+    }
+    int rc = allgather(h, h->d_recpack, (size_t)I * stride * 8);
+    if (rc) return rc;
+    std::vector<uint64_t> host((size_t)It * stride);
+    CU(cudaMemcpyAsync(host.data(), h->d_recpack, host.size() * 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    bool have = false;
+    const uint32_t first = h->p.comm ? 0 : h->ga.island_base;
+    const uint32_t last = h->p.comm ? It : h->ga.island_base + I;
+    for (uint32_t g = first; g < last; ++g) {
+        const uint64_t* e = host.data() + (size_t)g * stride;
+        double f;
+        memcpy(&f, e, 8);
+        const uint32_t gen = (uint32_t)(e[1] & 0xFFFFFFFFu);
+        const uint64_t* bits = e + 2;
+        if (!have || rec_better(f, bits, best->f, best->bits.data(), W) ||
+            (f == best->f && memcmp(bits, best->bits.data(), W * 8) == 0 && gen < best->gen)) {
+            best->f = f;
+            best->gen = gen;
+            best->bits.assign(bits, bits + W);
+            have = true;
+        }
+    }
+    return SPLIT_OK;
+}
+
+extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, split_best_t* best_out)
+{
+    if (!h || !best_out) return fail(SPLIT_E_INVAL, "split_ga_run: NULL argument");
+    CU(cudaSetDevice(h->device));
+    GaArgs& a = h->ga;
+    a.key0 = (uint32_t)seed;
+    a.key1 = (uint32_t)(seed >> 32);
+    const bool single = a.I_total == 1;
+    a.stall_in_kernel = single ? 1u : 0u;
+    h->stats = split_run_stats{};
+    CU(cudaMemsetAsync(a.rec_valid, 0, a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.cand_cnt, 0, 2 * a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.sel_cnt, 0, a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.ghist, 0, 3 * a.I * 256 * 4, h->stream));
+    CU(cudaEventRecord(h->ev[0], h->stream));
+    int rc = run_kernel(h, MODE_INIT, 0, 0);
+    if (rc) return rc;
+    CU(cudaEventRecord(h->ev[1], h->stream));
+    uint32_t gens_run = 0;
+    const uint32_t M = h->p.migration_interval;
+    if (single || M == 0) {
+        if (generations > 0) {
+            rc = run_kernel(h, MODE_RUN, 0, generations);
+            if (rc) return rc;
+        }
+        Ctl ctl;
+        CU(cudaMemcpyAsync(&ctl, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaStreamSynchronize(h->stream));
+        gens_run = generations > 0 ? ctl.gens_run : 0;
+        h->stats.general_selects = ctl.n_general;
+        h->stats.fast_selects = ctl.n_fast;
+    } else {
+        GlobalRec gr;
+        rc = global_record(h, &gr);
+        if (rc) return rc;
+        double f_improve = gr.f;
+        uint32_t last_improve = 0;
+        uint32_t g = 0;
+        while (g < generations) {
+            const uint32_t g1 = std::min<uint32_t>((g / M + 1) * M, generations);
+            rc = run_kernel(h, MODE_RUN, g, g1);
+            if (rc) return rc;
+            g = g1;
+            Ctl ctl;
+            CU(cudaMemcpyAsync(&ctl, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, h->stream));
+            CU(cudaStreamSynchronize(h->stream));
+            h->stats.general_selects += ctl.n_general;
+            h->stats.fast_selects += ctl.n_fast;
+            if (g % M != 0) break;   // g == generations, not a sync point
+            rc = global_record(h, &gr);
+            if (rc) return rc;
+            if (gr.f > f_improve) {
+                f_improve = gr.f;
+                last_improve = g;
+            }
+            if (h->p.stall_generations > 0 && g - last_improve >= h->p.stall_generations) break;
+            if (g < generations) {
+                rc = run_kernel(h, MODE_EXPORT, g, g);
+                if (rc) return rc;
+                rc = allgather(h, a.mig_bits, (size_t)a.I * a.K * h->W * 8);
+                if (rc) return rc;
+                rc = allgather(h, a.mig_f, (size_t)a.I * a.K * 8);
+                if (rc) return rc;
+                rc = run_kernel(h, MODE_IMPORT, g, g);
+                if (rc) return rc;
+            }
+        }
+        gens_run = g;
+    }
+    CU(cudaEventRecord(h->ev[2], h->stream));
+    GlobalRec best;
+    rc = global_record(h, &best);
+    if (rc) return rc;
+    // statistics of the best split
+    CU(cudaMemcpyAsync(h->d_bits1, best.bits.data(), h->W * 8, cudaMemcpyHostToDevice, h->stream));
+    CU(launch_eval_stats(h->ch, h->d_bits1, h->d_stats, h->d_statf, h->stream));
+    ++h->stats.launches;
+    int64_t st[5];
+    double fchk;
+    CU(cudaMemcpyAsync(st, h->d_stats, sizeof(st), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaMemcpyAsync(&fchk, h->d_statf, 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    CU(cudaEventElapsedTime(&h->stats.ms_total, h->ev[0], h->ev[2]));
+    CU(cudaEventElapsedTime(&h->stats.ms_loop, h->ev[1], h->ev[2]));
+    if (best_out->bits) memcpy(best_out->bits, best.bits.data(), h->W * 8);
+    best_out->fitness = best.f;
+    best_out->k = (uint32_t)st[0];
+    best_out->var_num = st[1];
+    best_out->s1 = (uint64_t)st[2];
+    best_out->s2 = (uint64_t)st[3];
+    best_out->overhead_ns = (uint64_t)st[4];
+    best_out->expected_wait_ns = st[2] > 0 ? (double)(uint64_t)st[3] / (2.0 * (double)(uint64_t)st[2]) : 0.0;
+    best_out->generation_found = best.gen;
+    best_out->generations_run = gens_run;
+    best_out->evaluations = (uint64_t)a.I * ((uint64_t)a.N + (uint64_t)gens_run * (a.N - a.E));
+    h->last_gen = gens_run;
+    h->have_pop = true;
+    if (fchk != best.f) return fail(SPLIT_E_STATE, "best record fitness mismatch (internal)");
+    return SPLIT_OK;
+}
+
+extern "C" int split_ga_population(split_ga_t* h, uint32_t island, uint64_t* bits_host, double* fit_host)
+{
+    if (!h) return fail(SPLIT_E_INVAL, "split_ga_population: NULL handle");
+    if (!h->have_pop) return fail(SPLIT_E_STATE, "no population: call split_ga_run first");
+    if (island >= h->ga.I) return fail(SPLIT_E_INVAL, "local island out of range");
+    CU(cudaSetDevice(h->device));
+    const uint32_t b = h->last_gen & 1u;
+    const size_t N = h->ga.N, W = h->W;
+    if (bits_host)
+        CU(cudaMemcpyAsync(bits_host, h->ga.pop[b] + island * N * W, N * W * 8, cudaMemcpyDeviceToHost, h->stream));
+    if (fit_host) CU(cudaMemcpyAsync(fit_host, h->ga.fit[b] + island * N, N * 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    return SPLIT_OK;
+}
+
+extern "C" int split_last_run_stats(const split_ga_t* h, split_run_stats* out)
+{
+    if (!h || !out) return fail(SPLIT_E_INVAL, "NULL argument");
+    *out = h->stats;
+    return SPLIT_OK;
+}
+
+// ------------------------------------------------------------------------
+// a10 — Algorithm 1 (greedy preemption), reading R12:
+// scanning from the tail, t_new passes t_i iff the types differ and
+// Ext_left(t_i)*Ext(t_i) > Ext_left(t_new)*Ext(t_new); it stops behind the
+// first t_i it does not pass, or reaches the head.  alpha and the waited
+// times cancel out of line 13's comparison.
+// ------------------------------------------------------------------------
+static bool req_ok(const split_request& r) { return r.ext_ns > 0 && r.ext_left_ns >= 0 && r.ext_left_ns <= r.ext_ns; }
+
+extern "C" int split_preempt_decide(const split_queue_state* q, uint32_t* insert_pos)
+{
+    if (!q || !insert_pos) return fail(SPLIT_E_INVAL, "split_preempt_decide: NULL argument");
+    if (!(q->alpha > 0.0) || !isfinite(q->alpha)) return fail(SPLIT_E_INVAL, "alpha must be > 0");
+    if (q->n > 0 && !q->queue) return fail(SPLIT_E_INVAL, "queue is NULL");
+    if (!req_ok(q->incoming)) return fail(SPLIT_E_INVAL, "incoming request: need ext > 0, 0 <= ext_left <= ext");
+    for (uint32_t i = 0; i < q->n; ++i)
+        if (!req_ok(q->queue[i])) return fail(SPLIT_E_INVAL, "queue[%u]: need ext > 0, 0 <= ext_left <= ext", i);
+    const __int128 w_new = (__int128)q->incoming.ext_left_ns * q->incoming.ext_ns;
+    for (uint32_t j = q->n; j-- > 0;) {
+        const split_request& t = q->queue[j];
+        if (t.type_id == q->incoming.type_id) { *insert_pos = j + 1; return SPLIT_OK; }
+        if ((__int128)t.ext_left_ns * t.ext_ns <= w_new) { *insert_pos = j + 1; return SPLIT_OK; }
+    }
+    *insert_pos = 0;
+    return SPLIT_OK;
+}
+
+// ------------------------------------------------------------------------
+// device self-tests
+// ------------------------------------------------------------------------
+extern "C" int split_selftest_philox(int device, const uint32_t* in, uint32_t n, uint32_t* out)
+{
+    if ((!in || !out) && n) return fail(SPLIT_E_INVAL, "NULL buffer");
+    if (n == 0) return SPLIT_OK;
+    CU(cudaSetDevice(device));
+    uint32_t *di = nullptr, *dout = nullptr;
+    CU(cudaMalloc(&di, (size_t)n * 24));
+    CU(cudaMalloc(&dout, (size_t)n * 16));
+    cudaError_t e = cudaMemcpy(di, in, (size_t)n * 24, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = launch_selftest_philox(di, n, dout, 0);
+    if (e == cudaSuccess) e = cudaMemcpy(out, dout, (size_t)n * 16, cudaMemcpyDeviceToHost);
+    cudaFree(di);
+    cudaFree(dout);
+    if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "selftest_philox: %s", cudaGetErrorString(e));
+    return SPLIT_OK;
+}
+
+extern "C" int split_selftest_dexp(int device, const double* in, uint32_t n, double* out)
+{
+    if ((!in || !out) && n) return fail(SPLIT_E_INVAL, "NULL buffer");
+    if (n == 0) return SPLIT_OK;
+    CU(cudaSetDevice(device));
+    double *di = nullptr, *dout = nullptr;
+    CU(cudaMalloc(&di, (size_t)n * 8));
+    CU(cudaMalloc(&dout, (size_t)n * 8));
+    cudaError_t e = cudaMemcpy(di, in, (size_t)n * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = launch_selftest_dexp(di, n, dout, 0);
+    if (e == cudaSuccess) e = cudaMemcpy(out, dout, (size_t)n * 8, cudaMemcpyDeviceToHost);
+    cudaFree(di);
+    cudaFree(dout);
+    if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "selftest_dexp: %s", cudaGetErrorString(e));
+    return SPLIT_OK;
+}

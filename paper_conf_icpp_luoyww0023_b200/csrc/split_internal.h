@@ -1,0 +1,84 @@
+// split_internal.h — device state and kernel launchers shared by split_host.cpp
+// and split_kernels.cu (product code; nothing here is shared with oracle/).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace splitga {
+
+constexpr uint32_t kMaxLocalIslands = 16;   // islands batched on one device
+constexpr uint32_t kMaxElite = 1024;        // E and K (v1 bound)
+constexpr uint32_t kCandCap = 2048;         // fast elite merge handles up to this many candidates
+constexpr uint32_t kMaxWords = 64;          // n_ops <= 4097
+constexpr uint32_t kBlock = 256;            // threads per CTA of the GA kernel
+
+enum Tag : uint32_t { TAG_INIT = 1, TAG_SELECT = 2, TAG_XOVER = 3, TAG_MUTATE = 4, TAG_REPAIR = 5 };
+enum Mode : uint32_t { MODE_INIT = 0, MODE_RUN = 1, MODE_EXPORT = 2, MODE_IMPORT = 3 };
+
+// device-resident control block (one per handle)
+struct Ctl {
+    uint32_t full;          // next SEL must use the general (radix) top-E path
+    uint32_t done;          // stall reached (single island, in-kernel)
+    uint32_t gens_run;      // generation reached by the last RUN segment
+    uint32_t last_improve;  // generation of the last strict improvement (single island)
+    double f_improve;       // record fitness at the last improvement
+    uint32_t n_general, n_fast;
+    uint32_t pad[2];
+};
+
+// Chain staged for the kernels: P[0..n] (u32, exclusive prefix of the latencies)
+// padded to a multiple of 4 words, then ovh[0..n-2] (u32) padded likewise.
+struct ChainDev {
+    const uint32_t* words;  // device
+    uint32_t n, W;
+    uint32_t p_words, o_words;  // padded lengths (multiples of 4)
+    uint32_t T;                 // == P[n]
+    uint32_t k_min, k_max;
+    uint64_t last_mask;         // valid bits of word W-1
+};
+
+// All device pointers and scalars the GA kernel needs (passed by value).
+struct GaArgs {
+    ChainDev ch;
+    uint32_t N, E, s, K;               // population, elites, tournament size, migrants
+    uint32_t I, island_base, I_total;  // local islands, first global island, all islands
+    uint32_t front_skip, stall;
+    uint64_t thr_c, thr_m;             // Bernoulli thresholds floor(p * 2^32)
+    uint32_t key0, key1;               // Philox key (seed lo, hi)
+    uint32_t mode, g_begin, g_end;     // MODE_*, generation range of a RUN segment
+    uint32_t stall_in_kernel;          // single global island: stall checked every generation
+    uint32_t sort_cap;                 // power of two, entries the leader can sort in smem
+    uint64_t* pop[2];                  // [I][N][W]
+    double* fit[2];                    // [I][N]
+    uint64_t* cand_key[2];             // [I][N]   candidates of generation g (parity g&1)
+    uint32_t* cand_idx[2];
+    uint32_t* cand_cnt;                // [2][I]
+    uint64_t* sel_key;                 // [I][kMaxElite] general-select / elite output
+    uint32_t* sel_idx;
+    uint32_t* sel_cnt;                 // [I]
+    uint64_t* tau;                     // [I] key of the worst elite of the current generation
+    uint32_t* ghist;                   // [3][I][256]
+    double* part_f;                    // [2][I][cpi] per-CTA best child
+    uint32_t* part_idx;
+    double* rec_f;                     // [I] island records
+    uint64_t* rec_bits;                // [I][W]
+    uint32_t* rec_gen;                 // [I]
+    uint32_t* rec_valid;               // [I]
+    uint64_t* mig_bits;                // [I_total][K][W]
+    double* mig_f;                     // [I_total][K]
+    Ctl* ctl;
+};
+
+// Launchers (split_kernels.cu).  Return cudaError_t of the launch.
+cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out,
+                              cudaStream_t st, int num_sms, uint64_t* launches);
+// Cooperative persistent GA kernel; grid = blocks_per_sm * num_sms.
+cudaError_t launch_ga(const GaArgs& a, cudaStream_t st, int num_sms, uint64_t* launches);
+size_t ga_smem_bytes(const GaArgs& a);
+int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err);
+cudaError_t launch_eval_stats(const ChainDev& ch, const uint64_t* bits, int64_t* stats_out /*[5]*/,
+                              double* f_out, cudaStream_t st);
+cudaError_t launch_selftest_philox(const uint32_t* in, uint32_t n, uint32_t* out, cudaStream_t st);
+cudaError_t launch_selftest_dexp(const double* in, uint32_t n, double* out, cudaStream_t st);
+
+}  // namespace splitga

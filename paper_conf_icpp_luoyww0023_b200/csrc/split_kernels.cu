@@ -1,0 +1,1185 @@
+// split_kernels.cu — sm_100a kernels of the GA split search (SPLIT, ICPP'23 §3.3).
+//
+// K1  eval_batch_kernel   a2: bitset -> (k, S1, S2, V, OV) exact integers -> Eq. 2 in FP64
+//                          (PAPER.md P@21101-21296).  Chain prefix/overheads staged into
+//                          shared memory with one TMA bulk copy (cp.async.bulk + mbarrier);
+//                          bitset tiles loaded with coalesced 128-bit loads per warp.
+// K2+ ga_kernel            cooperative persistent kernel, one launch per GA segment:
+//                          a1 init (Philox + Floyd), a3 elite top-E (radix select over the
+//                          96-bit (fitness key, ~index) order, or a single-CTA merge of the
+//                          previous elites with the few children that beat the worst elite),
+//                          a4-a7 breed (tournament, one-point crossover, one-bit mutation,
+//                          rank-select repair) fused with a2 eval of the children, a8 best
+//                          record + stall, a9 migration export/import.
+// Everything is integer / FP64 scalar work: no tensor cores (north_star).
+// Determinism: every random draw is Philox4x32-10 keyed on (seed) with counter
+// (global individual, generation, tag, draw/4) (R9), and every
+// reduction breaks ties by index or bitset, so results match the CPU oracle
+// bit for bit.
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <stdint.h>
+
+#include "split_internal.h"
+
+namespace cg = cooperative_groups;
+
+namespace splitga {
+
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+
+// ------------------------------------------------------------------------
+// Philox4x32-10 (Salmon et al., SC'11), multipliers/Weyl constants of the
+// Random123 reference.  Device-side implementation, independent of oracle/.
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint4 philox10(uint4 c, uint32_t k0, uint32_t k1)
+{
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = __umulhi(0xD2511F53u, c.x);
+        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = __umulhi(0xCD9E8D57u, c.z);
+        c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    return c;
+}
+
+__device__ __forceinline__ uint32_t lane_of(const uint4& v, uint32_t l)
+{
+    return l == 0 ? v.x : (l == 1 ? v.y : (l == 2 ? v.z : v.w));
+}
+
+// sequential draws d = 0, 1, ... of one (id, gen, tag) stream
+struct Draws {
+    uint32_t id, gen, tag, d, k0, k1;
+    uint4 blk;
+    __device__ __forceinline__ Draws(uint32_t id_, uint32_t gen_, uint32_t tag_, uint32_t k0_, uint32_t k1_)
+        : id(id_), gen(gen_), tag(tag_), d(0), k0(k0_), k1(k1_) {}
+    __device__ __forceinline__ uint32_t next()
+    {
+        if ((d & 3u) == 0) blk = philox10(make_uint4(id, gen, tag, d >> 2), k0, k1);
+        return lane_of(blk, (d++) & 3u);
+    }
+};
+
+// uniform integer in [0, m): floor(u * m / 2^32)
+__device__ __forceinline__ uint32_t below(uint32_t u, uint32_t m) { return __umulhi(u, m); }
+
+// ------------------------------------------------------------------------
+// dexp: exp by the fixed operation sequence of DESIGN.md R5'' (Cody-Waite
+// reduction, degree-13 Taylor polynomial in Horner form, RN(1/i!)).
+// ------------------------------------------------------------------------
+__device__ __forceinline__ double dexp_dev(double z)
+{
+    if (z > 710.0) return CUDART_INF;
+    if (z < -700.0) return 0.0;
+    const double j = rint(__dmul_rn(z, 0x1.71547652b82fep+0));
+    double r = __fma_rn(-j, 0x1.62e42fefa39efp-1, z);
+    r = __fma_rn(-j, 0x1.abc9e3b39803fp-56, r);
+    double p = 0x1.6124613a86d09p-33;           // 1/13!
+    p = __fma_rn(p, r, 0x1.1eed8eff8d898p-29);  // 1/12!
+    p = __fma_rn(p, r, 0x1.ae64567f544e4p-26);  // 1/11!
+    p = __fma_rn(p, r, 0x1.27e4fb7789f5cp-22);  // 1/10!
+    p = __fma_rn(p, r, 0x1.71de3a556c734p-19);  // 1/9!
+    p = __fma_rn(p, r, 0x1.a01a01a01a01ap-16);  // 1/8!
+    p = __fma_rn(p, r, 0x1.a01a01a01a01ap-13);  // 1/7!
+    p = __fma_rn(p, r, 0x1.6c16c16c16c17p-10);  // 1/6!
+    p = __fma_rn(p, r, 0x1.1111111111111p-7);   // 1/5!
+    p = __fma_rn(p, r, 0x1.5555555555555p-5);   // 1/4!
+    p = __fma_rn(p, r, 0x1.5555555555555p-3);   // 1/3!
+    p = __fma_rn(p, r, 0.5);
+    p = __fma_rn(p, r, 1.0);
+    p = __fma_rn(p, r, 1.0);
+    return ldexp(p, (int)j);
+}
+
+// Eq. 2 from the exact integer statistics (R5'):
+//   x = sigma/T = sqrt(V)/(k T),  y = overhead/m = (OV/T)/k,  f = -(e^(x-1) + e^(y-1))
+__device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, uint32_t T)
+{
+    const double Td = __uint2double_rn(T);
+    const double kd = __uint2double_rn(k);
+    const double x = __ddiv_rn(__dsqrt_rn(__ll2double_rn(V)), __dmul_rn(kd, Td));
+    const double y = __ddiv_rn(__ddiv_rn(__ull2double_rn(OV), Td), kd);
+    return -__dadd_rn(dexp_dev(__dsub_rn(x, 1.0)), dexp_dev(__dsub_rn(y, 1.0)));
+}
+
+// order-preserving u64 key of a fitness (larger f -> larger key)
+__device__ __forceinline__ uint64_t fkey(double f)
+{
+    const uint64_t u = (uint64_t)__double_as_longlong(f);
+    return (u >> 63) ? ~u : (u | 0x8000000000000000ull);
+}
+__device__ __forceinline__ double unkey(uint64_t k)
+{
+    const uint64_t u = (k >> 63) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
+    return __longlong_as_double((long long)u);
+}
+
+// ------------------------------------------------------------------------
+// Chain staging: one TMA bulk copy of P|ovh into shared memory.
+// ------------------------------------------------------------------------
+__device__ __forceinline__ void stage_chain(uint32_t* s_chain, const ChainDev& ch, uint64_t* mbar)
+{
+    const uint32_t bytes = (ch.p_words + ch.o_words) * 4u;   // multiple of 16
+    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(s_chain);
+        const uint32_t chunk = 32768u;
+        for (uint32_t off = 0; off < bytes; off += chunk) {
+            const uint32_t b = (bytes - off < chunk) ? (bytes - off) : chunk;
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst + off),
+                "l"((const char*)ch.words + off), "r"(b), "r"(bar)
+                : "memory");
+        }
+    }
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+            : "=r"(ok)
+            : "r"(bar)
+            : "memory");
+    }
+}
+
+// Walk the cuts of one candidate: words come from `get(w)` in ascending order.
+// Block j ends at cut c_j; t_j = P[c_j+1] - P[c_{j-1}+1] + ovh[c_{j-1}] (R3).
+struct Stats {
+    uint32_t k;
+    int64_t V;
+    uint64_t S1, S2, OV;
+};
+
+template <class Get>
+__device__ __forceinline__ double eval_walk(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO, Get get,
+                                            Stats* st)
+{
+    uint32_t cuts = 0;
+    for (uint32_t w = 0; w < ch.W; ++w) {
+        uint64_t v = get(w);
+        if (w == ch.W - 1) v &= ch.last_mask;
+        cuts += __popcll(v);
+    }
+    const uint32_t k = cuts + 1;
+    if (k < ch.k_min || k > ch.k_max) {
+        if (st) st->k = k;
+        return -CUDART_INF;
+    }
+    uint32_t startP = 0, prev_o = 0;
+    uint64_t S1 = 0, S2 = 0, OV = 0;
+    for (uint32_t w = 0; w < ch.W; ++w) {
+        uint64_t v = get(w);
+        if (w == ch.W - 1) v &= ch.last_mask;
+        while (v) {
+            const uint32_t p = w * 64u + (uint32_t)(__ffsll((long long)v) - 1);
+            v &= v - 1;
+            const uint32_t Pp = sP[p + 1];
+            const uint32_t t = Pp - startP + prev_o;
+            S1 += t;
+            S2 += (uint64_t)t * t;
+            prev_o = sO[p];
+            OV += prev_o;
+            startP = Pp;
+        }
+    }
+    const uint32_t t = ch.T - startP + prev_o;
+    S1 += t;
+    S2 += (uint64_t)t * t;
+    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);   // exact: V < 2^63 by the a0 guard
+    if (st) { st->k = k; st->V = V; st->S1 = S1; st->S2 = S2; st->OV = OV; }
+    return eq2(k, V, OV, ch.T);
+}
+
+// ------------------------------------------------------------------------
+// K1: split_eval_batch.  Each warp stages 32 rows (coalesced 128-bit loads)
+// into a padded shared tile (odd pitch: conflict-free row reads), then every
+// lane walks its own candidate.
+// ------------------------------------------------------------------------
+constexpr int kEvalWarps = 8;
+
+__global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
+                                                                     uint64_t n_cand, double* __restrict__ out)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint32_t* s_chain = (uint32_t*)smem;
+    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
+    uint64_t* s_tiles = mbar + 2;
+    const uint32_t W = ch.W;
+    const uint32_t pitch = W | 1u;
+    stage_chain(s_chain, ch, mbar);
+    const uint32_t* sP = s_chain;
+    const uint32_t* sO = s_chain + ch.p_words;
+
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint64_t* tile = s_tiles + (size_t)warp * 32u * pitch;
+    const uint64_t n_tiles = (n_cand + 31) / 32;
+    const uint64_t gw = (uint64_t)blockIdx.x * kEvalWarps + warp;
+    const uint64_t nw = (uint64_t)gridDim.x * kEvalWarps;
+    for (uint64_t t = gw; t < n_tiles; t += nw) {
+        const uint64_t row0 = t * 32;
+        const uint32_t rows = (uint32_t)((n_cand - row0) < 32 ? (n_cand - row0) : 32);
+        const uint64_t* src = bits + row0 * W;
+        const uint32_t nwords = rows * W;
+        if (rows == 32) {
+            const uint4* src4 = (const uint4*)src;        // 256*W bytes, 16-byte aligned
+            const uint32_t n4 = 16u * W;
+#pragma unroll 4
+            for (uint32_t j = lane; j < n4; j += 32) {
+                const uint4 v = __ldcs(src4 + j);
+                const uint32_t w0 = 2 * j, w1 = 2 * j + 1;
+                tile[(w0 / W) * pitch + (w0 % W)] = ((uint64_t)v.y << 32) | v.x;
+                tile[(w1 / W) * pitch + (w1 % W)] = ((uint64_t)v.w << 32) | v.z;
+            }
+        } else {
+            for (uint32_t j = lane; j < nwords; j += 32) tile[(j / W) * pitch + (j % W)] = __ldcs(src + j);
+        }
+        __syncwarp();
+        if (lane < rows) {
+            const uint64_t* my = tile + lane * pitch;
+            const double f = eval_walk(ch, sP, sO, [&](uint32_t w) { return my[w]; }, nullptr);
+            __stcs(out + row0 + lane, f);
+        }
+        __syncwarp();
+    }
+}
+
+// ------------------------------------------------------------------------
+// GA kernel helpers
+// ------------------------------------------------------------------------
+template <int WT>
+struct Row {
+    uint64_t w[WT];
+};
+
+template <int WT>
+__device__ __forceinline__ void row_load(Row<WT>& r, const uint64_t* src, uint32_t W)
+{
+#pragma unroll
+    for (int i = 0; i < WT; ++i) r.w[i] = (i < (int)W) ? src[i] : 0ull;
+}
+template <int WT>
+__device__ __forceinline__ void row_store(const Row<WT>& r, uint64_t* dst, uint32_t W)
+{
+#pragma unroll
+    for (int i = 0; i < WT; ++i)
+        if (i < (int)W) dst[i] = r.w[i];
+}
+template <int WT>
+__device__ __forceinline__ void row_xor_bit(Row<WT>& r, uint32_t p)
+{
+#pragma unroll
+    for (int i = 0; i < WT; ++i)
+        if ((uint32_t)i == (p >> 6)) r.w[i] ^= 1ull << (p & 63);
+}
+template <int WT>
+__device__ __forceinline__ bool row_get_bit(const Row<WT>& r, uint32_t p)
+{
+    bool b = false;
+#pragma unroll
+    for (int i = 0; i < WT; ++i)
+        if ((uint32_t)i == (p >> 6)) b = (r.w[i] >> (p & 63)) & 1ull;
+    return b;
+}
+__device__ __forceinline__ uint64_t word_mask(const ChainDev& ch, uint32_t w)
+{
+    return (w + 1 == ch.W) ? ch.last_mask : ~0ull;
+}
+template <int WT>
+__device__ __forceinline__ uint32_t row_popc(const Row<WT>& r, const ChainDev& ch)
+{
+    uint32_t c = 0;
+#pragma unroll
+    for (int i = 0; i < WT; ++i)
+        if (i < (int)ch.W) c += __popcll(r.w[i] & word_mask(ch, i));
+    return c;
+}
+
+// position of the r-th (0-based) set bit of m (r < popc(m))
+__device__ __forceinline__ uint32_t select_bit(uint64_t m, uint32_t r)
+{
+    uint32_t pos = 0;
+    uint32_t c = __popc((uint32_t)m);
+    if (r >= c) { r -= c; m >>= 32; pos += 32; }
+    uint32_t x = (uint32_t)m;
+    c = __popc(x & 0xFFFFu); if (r >= c) { r -= c; x >>= 16; pos += 16; }
+    c = __popc(x & 0xFFu);   if (r >= c) { r -= c; x >>= 8;  pos += 8; }
+    c = __popc(x & 0xFu);    if (r >= c) { r -= c; x >>= 4;  pos += 4; }
+    c = __popc(x & 0x3u);    if (r >= c) { r -= c; x >>= 2;  pos += 2; }
+    if (r >= (x & 1u)) pos += 1;
+    return pos;
+}
+
+// clear (set) the r-th set (unset) valid position, ascending order
+template <int WT>
+__device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch, uint32_t r, bool among_set)
+{
+    bool done = false;
+#pragma unroll
+    for (int i = 0; i < WT; ++i) {
+        if (i < (int)ch.W && !done) {
+            const uint64_t m = (among_set ? row.w[i] : ~row.w[i]) & word_mask(ch, i);
+            const uint32_t c = __popcll(m);
+            if (r < c) {
+                row.w[i] ^= 1ull << select_bit(m, r);
+                done = true;
+            } else {
+                r -= c;
+            }
+        }
+    }
+}
+
+template <int WT>
+__device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
+                                            const Row<WT>& r, Stats* st)
+{
+    return eval_walk(
+        ch, sP, sO,
+        [&](uint32_t w) {
+            uint64_t v = 0;
+#pragma unroll
+            for (int i = 0; i < WT; ++i)
+                if ((uint32_t)i == w) v = r.w[i];
+            return v;
+        },
+        st);
+}
+
+// best-record order: (f desc, bitset asc; word W-1 most significant)
+__device__ __forceinline__ bool rows_less(const uint64_t* a, const uint64_t* b, uint32_t W)
+{
+    for (int w = (int)W - 1; w >= 0; --w)
+        if (a[w] != b[w]) return a[w] < b[w];
+    return false;
+}
+__device__ __forceinline__ bool better_rec(double fa, uint32_t ia, double fb, uint32_t ib, const uint64_t* base,
+                                           uint32_t W)
+{
+    if (ia == NONE) return false;
+    if (ib == NONE) return true;
+    if (fa != fb) return fa > fb;
+    return rows_less(base + (size_t)ia * W, base + (size_t)ib * W, W);
+}
+
+struct BestRef {
+    double f;
+    uint32_t idx;
+};
+
+// block-wide best by (f desc, bits asc) over rows of `base`; all threads call.
+__device__ BestRef block_best(BestRef v, const uint64_t* base, uint32_t W, BestRef* scratch)
+{
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+#pragma unroll
+    for (int off = 16; off; off >>= 1) {
+        BestRef o;
+        o.f = __shfl_down_sync(0xFFFFFFFFu, v.f, off);
+        o.idx = __shfl_down_sync(0xFFFFFFFFu, v.idx, off);
+        if (lane + off < 32 && better_rec(o.f, o.idx, v.f, v.idx, base, W)) v = o;
+    }
+    if (lane == 0) scratch[warp] = v;
+    __syncthreads();
+    if (warp == 0) {
+        v = (lane < nwarps) ? scratch[lane] : BestRef{-CUDART_INF, NONE};
+#pragma unroll
+        for (int off = 16; off; off >>= 1) {
+            BestRef o;
+            o.f = __shfl_down_sync(0xFFFFFFFFu, v.f, off);
+            o.idx = __shfl_down_sync(0xFFFFFFFFu, v.idx, off);
+            if (lane + off < 32 && better_rec(o.f, o.idx, v.f, v.idx, base, W)) v = o;
+        }
+        if (lane == 0) scratch[32] = v;
+    }
+    __syncthreads();
+    const BestRef r = scratch[32];
+    __syncthreads();
+    return r;
+}
+
+// composite ranking order (key desc, idx asc)
+__device__ __forceinline__ bool comp_gt(uint64_t ka, uint32_t ia, uint64_t kb, uint32_t ib)
+{
+    return ka > kb || (ka == kb && ia < ib);
+}
+
+// bitonic sort of n (power of two) entries in shared memory, descending composite
+__device__ void bitonic_desc(uint64_t* k, uint32_t* ix, uint32_t n)
+{
+    for (uint32_t size = 2; size <= n; size <<= 1) {
+        for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+            __syncthreads();
+            for (uint32_t t = threadIdx.x; t < n / 2; t += blockDim.x) {
+                const uint32_t lo = 2 * t - (t & (stride - 1));
+                const uint32_t hi = lo + stride;
+                const bool up = (lo & size) == 0;
+                const bool gt = comp_gt(k[lo], ix[lo], k[hi], ix[hi]);
+                if (gt != up) {
+                    const uint64_t tk = k[lo]; k[lo] = k[hi]; k[hi] = tk;
+                    const uint32_t ti = ix[lo]; ix[lo] = ix[hi]; ix[hi] = ti;
+                }
+            }
+        }
+    }
+    __syncthreads();
+}
+
+__device__ __forceinline__ uint32_t next_pow2(uint32_t x)
+{
+    uint32_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+// warp-aggregated append of (key, idx) when pred
+__device__ __forceinline__ void append_if(bool pred, uint32_t* cnt, uint64_t* keys, uint32_t* idxs, uint64_t key,
+                                          uint32_t idx)
+{
+    const unsigned act = __activemask();
+    const unsigned m = __ballot_sync(act, pred);
+    if (!m) return;
+    const uint32_t lane = threadIdx.x & 31u;
+    const int leader = __ffs(act) - 1;
+    uint32_t base = 0;
+    if ((int)lane == leader) base = atomicAdd(cnt, (uint32_t)__popc(m));
+    base = __shfl_sync(act, base, leader);
+    if (pred) {
+        const uint32_t r = __popc(m & ((1u << lane) - 1u));
+        keys[base + r] = key;
+        idxs[base + r] = idx;
+    }
+}
+
+// ------------------------------------------------------------------------
+// Shared-memory layout of the GA kernel
+// ------------------------------------------------------------------------
+struct SelState {
+    uint64_t ph;     // resolved prefix of the 96-bit composite (high 64 bits)
+    uint32_t pl;     // resolved prefix (low 32 bits)
+    uint32_t d;      // resolved digits (0..12)
+    uint32_t need;   // elements still to take from the threshold bin
+    uint32_t done;
+};
+
+struct Smem {
+    uint32_t* chain;
+    uint64_t* mbar;
+    uint32_t* hist;       // [I][256]
+    SelState* sel;        // [I]
+    BestRef* scratch;     // [33]
+    uint64_t* skey;       // [sort_cap]
+    uint32_t* sidx;       // [sort_cap]
+    uint64_t* ekey;       // [kMaxElite]
+};
+
+__host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
+
+__host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Smem* s)
+{
+    size_t off = 0;
+    auto take = [&](size_t bytes) { size_t o = off; off = align16(off + bytes); return base + o; };
+    uint8_t* p;
+    p = take((size_t)(a.ch.p_words + a.ch.o_words) * 4); if (s) s->chain = (uint32_t*)p;
+    p = take(16); if (s) s->mbar = (uint64_t*)p;
+    p = take((size_t)a.I * 256 * 4); if (s) s->hist = (uint32_t*)p;
+    p = take((size_t)a.I * sizeof(SelState)); if (s) s->sel = (SelState*)p;
+    p = take(33 * sizeof(BestRef)); if (s) s->scratch = (BestRef*)p;
+    p = take((size_t)a.sort_cap * 8); if (s) s->skey = (uint64_t*)p;
+    p = take((size_t)a.sort_cap * 4); if (s) s->sidx = (uint32_t*)p;
+    p = take((size_t)kMaxElite * 8); if (s) s->ekey = (uint64_t*)p;
+    return off;
+}
+
+// composite of element i of an island: desc order (elite/export) -> (key, ~idx);
+// worst order (import) -> (~key, idx).  Larger composite = selected first.
+__device__ __forceinline__ void composite(double f, uint32_t i, bool worst, uint64_t& hi, uint32_t& lo)
+{
+    const uint64_t k = fkey(f);
+    hi = worst ? ~k : k;
+    lo = worst ? i : ~i;
+}
+
+__device__ __forceinline__ bool sel_match(uint64_t hi, uint32_t lo, const SelState& s)
+{
+    if (s.d == 0) return true;
+    if (s.d <= 8) return (hi >> (64 - 8 * s.d)) == s.ph;
+    if (hi != s.ph) return false;
+    const uint32_t dl = s.d - 8;
+    return (dl == 4 ? lo : (lo >> (32 - 8 * dl))) == s.pl;
+}
+__device__ __forceinline__ uint32_t sel_digit(uint64_t hi, uint32_t lo, uint32_t d)
+{
+    return d < 8 ? (uint32_t)(hi >> (56 - 8 * d)) & 0xFFu : (lo >> (24 - 8 * (d - 8))) & 0xFFu;
+}
+__device__ __forceinline__ bool sel_selected(uint64_t hi, uint32_t lo, const SelState& s)
+{
+    if (s.d == 0) return true;
+    if (s.d <= 8) return (hi >> (64 - 8 * s.d)) >= s.ph;
+    if (hi != s.ph) return hi > s.ph;
+    const uint32_t dl = s.d - 8;
+    return (dl == 4 ? lo : (lo >> (32 - 8 * dl))) >= s.pl;
+}
+
+// General top-Ksel per local island by 96-bit radix select (MSB first, 8-bit
+// digits), all CTAs cooperating with grid barriers.  Output (unsorted):
+// sel_key/sel_idx[i][0..Ksel) with sel_cnt[i] == Ksel.  fit: [I][N].
+__device__ void general_select(const GaArgs& a, const double* fit, uint32_t Ksel, bool worst, const Smem& sm,
+                               cg::grid_group& grid)
+{
+    const uint32_t I = a.I, N = a.N;
+    for (uint32_t i = threadIdx.x; i < I; i += blockDim.x) {
+        SelState s;
+        s.ph = 0; s.pl = 0; s.d = 0; s.need = Ksel;
+        s.done = (Ksel >= N) || (Ksel == 0);
+        sm.sel[i] = s;
+    }
+    __syncthreads();
+    const uint64_t total = (uint64_t)I * N;
+    const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t gstride = (uint64_t)gridDim.x * blockDim.x;
+    uint32_t pass = 0;
+    for (;;) {
+        bool pending = false;
+        for (uint32_t i = 0; i < I; ++i) pending |= !sm.sel[i].done;
+        if (!pending) break;
+        uint32_t* gh = a.ghist + (size_t)(pass % 3) * I * 256;
+        for (uint32_t j = threadIdx.x; j < I * 256; j += blockDim.x) sm.hist[j] = 0;
+        __syncthreads();
+        for (uint64_t e = gtid; e < total; e += gstride) {
+            const uint32_t i = (uint32_t)(e / N), idx = (uint32_t)(e % N);
+            const SelState& s = sm.sel[i];
+            if (s.done) continue;
+            uint64_t hi; uint32_t lo;
+            composite(fit[e], idx, worst, hi, lo);
+            if (sel_match(hi, lo, s)) atomicAdd(&sm.hist[i * 256 + sel_digit(hi, lo, s.d)], 1u);
+        }
+        __syncthreads();
+        for (uint32_t j = threadIdx.x; j < I * 256; j += blockDim.x)
+            if (sm.hist[j]) atomicAdd(&gh[j], sm.hist[j]);
+        if (blockIdx.x == 0) {
+            uint32_t* z = a.ghist + (size_t)((pass + 1) % 3) * I * 256;
+            for (uint32_t j = threadIdx.x; j < I * 256; j += blockDim.x) z[j] = 0;
+        }
+        grid.sync();
+        // every CTA derives the same decision from the global histogram
+        if (threadIdx.x < 32) {
+            for (uint32_t i = 0; i < I; ++i) {
+                SelState s = sm.sel[i];
+                if (s.done) continue;
+                // lane l owns bins 255-8l .. 248-8l (descending)
+                const uint32_t lane = threadIdx.x;
+                uint32_t c[8], sum = 0;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) { c[q] = __ldcg(&gh[i * 256 + 255 - 8 * lane - q]); sum += c[q]; }
+                // exclusive prefix over lanes (descending bins)
+                uint32_t incl = sum;
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, incl, off);
+                    if (lane >= (uint32_t)off) incl += o;
+                }
+                const uint32_t excl = incl - sum;
+                const bool mine = excl < s.need && incl >= s.need;
+                const unsigned who = __ballot_sync(0xFFFFFFFFu, mine);
+                const int src = __ffs(who) - 1;
+                uint32_t bin = 0, cnt = 0, before = 0;
+                if (mine) {
+                    uint32_t acc = excl;
+                    for (int q = 0; q < 8; ++q) {
+                        if (acc + c[q] >= s.need) { bin = 255 - 8 * lane - q; cnt = c[q]; before = acc; break; }
+                        acc += c[q];
+                    }
+                }
+                bin = __shfl_sync(0xFFFFFFFFu, bin, src);
+                cnt = __shfl_sync(0xFFFFFFFFu, cnt, src);
+                before = __shfl_sync(0xFFFFFFFFu, before, src);
+                if (lane == 0) {
+                    s.need -= before;
+                    if (s.d < 8) s.ph = (s.ph << 8) | bin;
+                    else s.pl = (s.pl << 8) | bin;
+                    s.d += 1;
+                    if (cnt == s.need || s.d == 12) s.done = 1;
+                    sm.sel[i] = s;
+                }
+                __syncwarp();
+            }
+        }
+        __syncthreads();
+        ++pass;
+    }
+    // compaction: exactly Ksel per island satisfy sel_selected
+    for (uint64_t e = gtid; e < total; e += gstride) {
+        const uint32_t i = (uint32_t)(e / N), idx = (uint32_t)(e % N);
+        const SelState s = sm.sel[i];
+        const double f = fit[e];
+        uint64_t hi; uint32_t lo;
+        composite(f, idx, worst, hi, lo);
+        const bool take = (Ksel > 0) && sel_selected(hi, lo, s);
+        if (take) {
+            const uint32_t slot = atomicAdd(&a.sel_cnt[i], 1u);
+            a.sel_key[(size_t)i * kMaxElite + slot] = fkey(f);
+            a.sel_idx[(size_t)i * kMaxElite + slot] = idx;
+        }
+    }
+    grid.sync();
+    if (blockIdx.x == 0) {
+        for (uint32_t j = threadIdx.x; j < 3 * I * 256; j += blockDim.x) a.ghist[j] = 0;
+    }
+}
+
+// Leader CTA: sort the general-select output of island i in smem (ranking
+// order, or worst order) and leave it in sm.skey/sm.sidx[0..Ksel).
+__device__ void leader_sort_selected(const GaArgs& a, uint32_t i, uint32_t Ksel, bool worst, const Smem& sm)
+{
+    const uint32_t P2 = next_pow2(Ksel < 2 ? 2 : Ksel);
+    for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+        if (j < Ksel) {
+            const uint64_t k = a.sel_key[(size_t)i * kMaxElite + j];
+            const uint32_t x = a.sel_idx[(size_t)i * kMaxElite + j];
+            sm.skey[j] = worst ? ~k : k;
+            sm.sidx[j] = worst ? ~x : x;
+        } else {
+            sm.skey[j] = 0;
+            sm.sidx[j] = NONE;
+        }
+    }
+    bitonic_desc(sm.skey, sm.sidx, P2);
+    if (worst)
+        for (uint32_t j = threadIdx.x; j < Ksel; j += blockDim.x) { sm.skey[j] = ~sm.skey[j]; sm.sidx[j] = ~sm.sidx[j]; }
+    __syncthreads();
+    if (threadIdx.x == 0) a.sel_cnt[i] = 0;
+}
+
+// Leader CTA: record update of island i from the per-CTA partial bests of
+// generation g (rows in pop_g), and the single-island stall rule (R11).
+__device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t parity, uint32_t cpi,
+                              const uint64_t* pop_g, const Smem& sm)
+{
+    const uint32_t W = a.ch.W;
+    const uint64_t* base = pop_g + (size_t)i * a.N * W;
+    BestRef v{-CUDART_INF, NONE};
+    const double* pf = a.part_f + ((size_t)parity * a.I + i) * cpi;
+    const uint32_t* pi = a.part_idx + ((size_t)parity * a.I + i) * cpi;
+    for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x) {
+        const BestRef o{pf[j], pi[j]};
+        if (better_rec(o.f, o.idx, v.f, v.idx, base, W)) v = o;
+    }
+    v = block_best(v, base, W, sm.scratch);
+    if (threadIdx.x == 0) {
+        bool upd = false;
+        if (v.idx != NONE) {
+            if (!a.rec_valid[i]) upd = true;
+            else if (v.f != a.rec_f[i]) upd = v.f > a.rec_f[i];
+            else upd = rows_less(base + (size_t)v.idx * W, a.rec_bits + (size_t)i * W, W);
+        }
+        if (upd) {
+            a.rec_f[i] = v.f;
+            a.rec_gen[i] = g;
+            a.rec_valid[i] = 1;
+            for (uint32_t w = 0; w < W; ++w) a.rec_bits[(size_t)i * W + w] = base[(size_t)v.idx * W + w];
+        }
+        if (a.stall_in_kernel && i == 0) {
+            Ctl* c = a.ctl;
+            if (g == 0) {
+                c->f_improve = a.rec_f[0];
+                c->last_improve = 0;
+            } else {
+                if (a.rec_f[0] > c->f_improve) { c->f_improve = a.rec_f[0]; c->last_improve = g; }
+                if (a.stall > 0 && g - c->last_improve >= a.stall) c->done = 1;
+            }
+        }
+    }
+    __syncthreads();
+}
+
+// ------------------------------------------------------------------------
+// Breed (a4-a7 + fused a2) for one pair of children of island i.
+// ------------------------------------------------------------------------
+template <int WT>
+__device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, uint32_t g, const double* fit)
+{
+    uint32_t best = 0;
+    double bf = 0.0;
+    for (uint32_t d = 0; d < a.s; d += 4) {
+        const uint4 r = philox10(make_uint4(gid, g, TAG_SELECT, d >> 2), a.key0, a.key1);
+        uint32_t ids[4];
+        double fs[4];
+#pragma unroll
+        for (int l = 0; l < 4; ++l) {
+            ids[l] = below(lane_of(r, l), a.N);
+            fs[l] = (d + l < a.s) ? __ldcg(fit + ids[l]) : 0.0;
+        }
+#pragma unroll
+        for (int l = 0; l < 4; ++l) {
+            if (d + l >= a.s) break;
+            if ((d + l) == 0 || fs[l] > bf || (fs[l] == bf && ids[l] < best)) { best = ids[l]; bf = fs[l]; }
+        }
+    }
+    return best;
+}
+
+template <int WT>
+__device__ __forceinline__ void repair(const GaArgs& a, Row<WT>& row, uint32_t gid, uint32_t g)
+{
+    const ChainDev& ch = a.ch;
+    uint32_t c = row_popc(row, ch);
+    if (c + 1 >= ch.k_min && c + 1 <= ch.k_max) return;
+    Draws dr(gid, g, TAG_REPAIR, a.key0, a.key1);
+    const uint32_t npos = ch.n - 1;
+    while (c > ch.k_max - 1) {
+        row_toggle_rank(row, ch, below(dr.next(), c), true);
+        --c;
+    }
+    while (c < ch.k_min - 1) {
+        row_toggle_rank(row, ch, below(dr.next(), npos - c), false);
+        ++c;
+    }
+}
+
+template <int WT>
+__device__ __forceinline__ void init_row(const GaArgs& a, Row<WT>& row, uint32_t gid)
+{
+#pragma unroll
+    for (int i = 0; i < WT; ++i) row.w[i] = 0;
+    Draws dr(gid, 0, TAG_INIT, a.key0, a.key1);
+    const uint32_t k = a.ch.k_min + below(dr.next(), a.ch.k_max - a.ch.k_min + 1);
+    const uint32_t f = a.front_skip, m = a.ch.n - 1 - f;
+    for (uint32_t j = m - (k - 1); j < m; ++j) {
+        const uint32_t r = below(dr.next(), j + 1);
+        const uint32_t p = row_get_bit(row, f + r) ? f + j : f + r;
+        row_xor_bit(row, p);
+    }
+}
+
+// per-thread running best child, (f desc, bits asc); rows already in pop_n
+template <int WT>
+__device__ __forceinline__ void track_best(BestRef& b, double f, uint32_t idx, const Row<WT>& r,
+                                           const uint64_t* pop_island, uint32_t W)
+{
+    if (b.idx == NONE || f > b.f) { b.f = f; b.idx = idx; return; }
+    if (f < b.f) return;
+    const uint64_t* o = pop_island + (size_t)b.idx * W;
+    for (int w = (int)W - 1; w >= 0; --w) {
+        uint64_t mine = 0;
+#pragma unroll
+        for (int i = 0; i < WT; ++i)
+            if (i == w) mine = r.w[i];
+        if (mine != o[w]) {
+            if (mine < o[w]) { b.f = f; b.idx = idx; }
+            return;
+        }
+    }
+}
+
+template <int WT>
+__device__ __forceinline__ void breed_pair(const GaArgs& a, uint32_t i, uint32_t q, uint32_t g, const uint64_t* popc,
+                                           const double* fitc, uint64_t* popn, double* fitn, const uint32_t* sP,
+                                           const uint32_t* sO, uint64_t tau, uint32_t* ccnt, uint64_t* ckey,
+                                           uint32_t* cidx, BestRef& best)
+{
+    const ChainDev& ch = a.ch;
+    const uint32_t W = ch.W, N = a.N;
+    const uint32_t c0 = a.E + 2 * q;
+    const uint32_t gid0 = (a.island_base + i) * N + c0;
+    const uint32_t pa = tournament<WT>(a, gid0, g, fitc);
+    const uint32_t pb = tournament<WT>(a, gid0 + 1, g, fitc);
+    Row<WT> A, B;
+    row_load(A, popc + (size_t)pa * W, W);
+    row_load(B, popc + (size_t)pb * W, W);
+    const uint4 rx = philox10(make_uint4(gid0, g, TAG_XOVER, 0), a.key0, a.key1);
+    if ((uint64_t)rx.x < a.thr_c && ch.n >= 3) {
+        const uint32_t x = 1 + below(rx.y, ch.n - 2);   // positions < x from the first parent
+#pragma unroll
+        for (int w = 0; w < WT; ++w) {
+            const uint32_t lo = 64u * w;
+            const uint64_t m = (x >= lo + 64) ? ~0ull : (x <= lo ? 0ull : ((1ull << (x - lo)) - 1));
+            const uint64_t a0 = A.w[w], b0 = B.w[w];
+            A.w[w] = (a0 & m) | (b0 & ~m);
+            B.w[w] = (b0 & m) | (a0 & ~m);
+        }
+    }
+    // a6 mutation, a7 repair, a2 eval of each child (children c0 = A, c0+1 = B)
+    auto finish = [&](Row<WT>& ch_row, uint32_t h) {
+        const uint32_t gid = gid0 + h;
+        const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);
+        if ((uint64_t)rm.x < a.thr_m) row_xor_bit(ch_row, below(rm.y, ch.n - 1));
+        repair(a, ch_row, gid, g);
+        const double f = eval_regs(ch, sP, sO, ch_row, nullptr);
+        const uint32_t slot = c0 + h;
+        row_store(ch_row, popn + (size_t)slot * W, W);
+        fitn[slot] = f;
+        append_if(fkey(f) > tau, ccnt, ckey, cidx, fkey(f), slot);
+        track_best(best, f, slot, ch_row, popn, W);
+    };
+    finish(A, 0);
+    finish(B, 1);
+}
+
+// ------------------------------------------------------------------------
+// The cooperative persistent GA kernel
+// ------------------------------------------------------------------------
+template <int WT>
+__global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    Smem sm;
+    smem_layout(a, smem, &sm);
+    cg::grid_group grid = cg::this_grid();
+    stage_chain(sm.chain, a.ch, sm.mbar);
+    const uint32_t* sP = sm.chain;
+    const uint32_t* sO = sm.chain + a.ch.p_words;
+    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I;
+    const uint32_t cpi = gridDim.x / I;                 // CTAs per island
+    const uint32_t my_island = blockIdx.x / cpi;
+    const uint32_t my_local = blockIdx.x % cpi;
+    const bool worker = my_island < I;
+
+    if (a.mode == MODE_INIT) {
+        // a1: generation 0 into buffer 0 (all N individuals), partials into parity 0
+        if (worker) {
+            const uint32_t i = my_island;
+            uint64_t* pop = a.pop[0] + (size_t)i * N * W;
+            double* fit = a.fit[0] + (size_t)i * N;
+            BestRef best{-CUDART_INF, NONE};
+            for (uint32_t c = my_local * blockDim.x + threadIdx.x; c < N; c += cpi * blockDim.x) {
+                Row<WT> r;
+                init_row(a, r, (a.island_base + i) * N + c);
+                const double f = eval_regs(a.ch, sP, sO, r, nullptr);
+                row_store(r, pop + (size_t)c * W, W);
+                fit[c] = f;
+                track_best(best, f, c, r, pop, W);
+            }
+            __syncthreads();
+            best = block_best(best, pop, W, sm.scratch);
+            if (threadIdx.x == 0) {
+                a.part_f[(size_t)i * cpi + my_local] = best.f;
+                a.part_idx[(size_t)i * cpi + my_local] = best.idx;
+            }
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            a.ctl->full = 1;
+            a.ctl->done = 0;
+            a.ctl->gens_run = 0;
+            a.ctl->n_general = 0;
+            a.ctl->n_fast = 0;
+        }
+        grid.sync();
+        if (blockIdx.x < I) leader_record(a, blockIdx.x, 0, 0, cpi, a.pop[0], sm);
+        return;
+    }
+
+    if (a.mode == MODE_EXPORT || a.mode == MODE_IMPORT) {
+        const uint32_t g = a.g_begin, cur = g & 1u;
+        const bool worst = a.mode == MODE_IMPORT;
+        general_select(a, a.fit[cur], a.K, worst, sm, grid);
+        if (blockIdx.x < I) {
+            const uint32_t i = blockIdx.x;
+            leader_sort_selected(a, i, a.K, worst, sm);
+            uint64_t* pop = a.pop[cur] + (size_t)i * N * W;
+            double* fit = a.fit[cur] + (size_t)i * N;
+            if (!worst) {
+                // export the island's top-K (rows + fitness) to its slot of the gather buffer
+                const size_t gi = a.island_base + i;
+                for (uint32_t j = threadIdx.x; j < a.K * W; j += blockDim.x) {
+                    const uint32_t r = j / W, w = j % W;
+                    a.mig_bits[(gi * a.K + r) * W + w] = pop[(size_t)sm.sidx[r] * W + w];
+                }
+                for (uint32_t r = threadIdx.x; r < a.K; r += blockDim.x) a.mig_f[gi * a.K + r] = fit[sm.sidx[r]];
+            } else {
+                // worst slots in sidx[0..K); foreign migrants sorted by (f desc, source asc, rank asc)
+                uint32_t* worst_slot = (uint32_t*)sm.ekey;   // K <= kMaxElite u32 fit in ekey
+                for (uint32_t r = threadIdx.x; r < a.K; r += blockDim.x) worst_slot[r] = sm.sidx[r];
+                __syncthreads();
+                const uint32_t gi = a.island_base + i;
+                const uint32_t nf = (a.I_total - 1) * a.K;
+                const uint32_t P2 = next_pow2(nf < 2 ? 2 : nf);
+                for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+                    if (j < nf) {
+                        const uint32_t src = j / a.K, r = j % a.K;
+                        const uint32_t gsrc = src < gi ? src : src + 1;   // skip own island
+                        const uint32_t e = gsrc * a.K + r;
+                        sm.skey[j] = fkey(a.mig_f[e]);
+                        sm.sidx[j] = e;
+                    } else {
+                        sm.skey[j] = 0;
+                        sm.sidx[j] = NONE;
+                    }
+                }
+                bitonic_desc(sm.skey, sm.sidx, P2);
+                const uint32_t take = a.K < nf ? a.K : nf;
+                for (uint32_t j = threadIdx.x; j < take * W; j += blockDim.x) {
+                    const uint32_t r = j / W, w = j % W;
+                    pop[(size_t)worst_slot[r] * W + w] = a.mig_bits[(size_t)sm.sidx[r] * W + w];
+                }
+                for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) fit[worst_slot[r]] = a.mig_f[sm.sidx[r]];
+                __syncthreads();
+                // record update with the received migrants (R19)
+                BestRef v{-CUDART_INF, NONE};
+                for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) {
+                    const BestRef o{fit[worst_slot[r]], worst_slot[r]};
+                    if (better_rec(o.f, o.idx, v.f, v.idx, pop, W)) v = o;
+                }
+                v = block_best(v, pop, W, sm.scratch);
+                if (threadIdx.x == 0 && v.idx != NONE) {
+                    bool upd = !a.rec_valid[i];
+                    if (!upd) upd = (v.f != a.rec_f[i]) ? (v.f > a.rec_f[i])
+                                                         : rows_less(pop + (size_t)v.idx * W, a.rec_bits + (size_t)i * W, W);
+                    if (upd) {
+                        a.rec_f[i] = v.f;
+                        a.rec_gen[i] = g;
+                        a.rec_valid[i] = 1;
+                        for (uint32_t w = 0; w < W; ++w) a.rec_bits[(size_t)i * W + w] = pop[(size_t)v.idx * W + w];
+                    }
+                }
+                // the children's partial bests of this generation may point at replaced slots
+                for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x)
+                    a.part_idx[((size_t)cur * I + i) * cpi + j] = NONE;
+                if (threadIdx.x == 0 && i == 0) a.ctl->full = 1;
+            }
+        }
+        return;
+    }
+
+    // MODE_RUN: generations [g_begin, g_end)
+    uint32_t g = a.g_begin;
+    for (; g < a.g_end; ++g) {
+        const uint32_t cur = g & 1u, nxt = cur ^ 1u;
+        const uint64_t* popc_all = a.pop[cur];
+        // ---- phase S: elites of generation g (a3) + record/stall of generation g (a8)
+        bool general = a.ctl->full != 0;
+        if (!general && E > 0)
+            for (uint32_t i = 0; i < I; ++i) general |= __ldcg(&a.cand_cnt[cur * I + i]) > kCandCap;
+        general = general && E > 0;
+        if (general) general_select(a, a.fit[cur], E, false, sm, grid);
+        if (blockIdx.x < I) {
+            const uint32_t i = blockIdx.x;
+            leader_record(a, i, g, cur, cpi, popc_all, sm);
+            const uint64_t* popc = popc_all + (size_t)i * N * W;
+            const double* fitc = a.fit[cur] + (size_t)i * N;
+            if (E > 0) {
+                if (general) {
+                    leader_sort_selected(a, i, E, false, sm);
+                } else {
+                    // fast path: previous elites (slots 0..E-1, ranked) merged with the
+                    // children that beat the worst of them (candidates, key > tau)
+                    const uint32_t C = a.cand_cnt[cur * I + i];
+                    const uint32_t P2 = next_pow2(C < 2 ? 2 : C);
+                    const uint64_t* ck = a.cand_key[cur] + (size_t)i * N;
+                    const uint32_t* cx = a.cand_idx[cur] + (size_t)i * N;
+                    for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+                        sm.skey[j] = j < C ? ck[j] : 0ull;
+                        sm.sidx[j] = j < C ? cx[j] : NONE;
+                    }
+                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) sm.ekey[r] = fkey(fitc[r]);
+                    bitonic_desc(sm.skey, sm.sidx, P2);
+                    // merged rank of elite r: r + #(candidates with key > ekey[r]);
+                    // of candidate j: j + #(elites with key >= ckey[j])  (elites win ties: lower index)
+                    uint64_t* outk = a.sel_key + (size_t)i * kMaxElite;
+                    uint32_t* outx = a.sel_idx + (size_t)i * kMaxElite;
+                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+                        const uint64_t k = sm.ekey[r];
+                        uint32_t lo = 0, hi = C;    // first j with skey[j] <= k
+                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.skey[mid] > k) lo = mid + 1; else hi = mid; }
+                        const uint32_t rank = r + lo;
+                        if (rank < E) { outk[rank] = k; outx[rank] = r; }
+                    }
+                    for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
+                        const uint64_t k = sm.skey[j];
+                        uint32_t lo = 0, hi = E;    // first r with ekey[r] < k
+                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.ekey[mid] >= k) lo = mid + 1; else hi = mid; }
+                        const uint32_t rank = j + lo;
+                        if (rank < E) { outk[rank] = k; outx[rank] = sm.sidx[j]; }
+                    }
+                    __syncthreads();
+                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) { sm.skey[r] = outk[r]; sm.sidx[r] = outx[r]; }
+                    __syncthreads();
+                }
+                // copy the elites in rank order to slots 0..E-1 of generation g+1 (R18)
+                uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
+                double* fitn = a.fit[nxt] + (size_t)i * N;
+                for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
+                    const uint32_t r = j / W, w = j % W;
+                    popn[(size_t)r * W + w] = popc[(size_t)sm.sidx[r] * W + w];
+                }
+                for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(sm.skey[r]);
+                if (threadIdx.x == 0) a.tau[i] = sm.skey[E - 1];
+            } else if (threadIdx.x == 0) {
+                a.tau[i] = ~0ull;    // no elites: no candidate list
+            }
+            if (threadIdx.x == 0) {
+                a.cand_cnt[nxt * I + i] = 0;
+                if (i == 0) { if (general) a.ctl->n_general++; else a.ctl->n_fast++; }
+            }
+        }
+        grid.sync();
+        if (__ldcg(&a.ctl->done)) break;
+        if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;
+        // ---- phase B: children of generation g+1 (a4-a7 + a2)
+        if (worker) {
+            const uint32_t i = my_island;
+            const uint64_t* popc = popc_all + (size_t)i * N * W;
+            const double* fitc = a.fit[cur] + (size_t)i * N;
+            uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
+            double* fitn = a.fit[nxt] + (size_t)i * N;
+            const uint64_t tau = __ldcg(&a.tau[i]);
+            uint32_t* ccnt = a.cand_cnt + nxt * I + i;
+            uint64_t* ckey = a.cand_key[nxt] + (size_t)i * N;
+            uint32_t* cidx = a.cand_idx[nxt] + (size_t)i * N;
+            const uint32_t pairs = (N - E) / 2;
+            BestRef best{-CUDART_INF, NONE};
+            for (uint32_t q = my_local * blockDim.x + threadIdx.x; q < pairs; q += cpi * blockDim.x)
+                breed_pair<WT>(a, i, q, g, popc, fitc, popn, fitn, sP, sO, tau, ccnt, ckey, cidx, best);
+            __syncthreads();
+            best = block_best(best, popn, W, sm.scratch);
+            if (threadIdx.x == 0) {
+                a.part_f[((size_t)nxt * I + i) * cpi + my_local] = best.f;
+                a.part_idx[((size_t)nxt * I + i) * cpi + my_local] = best.idx;
+            }
+        }
+        grid.sync();
+    }
+    if (g == a.g_end) {
+        // record (and stall) of the last generation of the segment
+        if (blockIdx.x < I) leader_record(a, blockIdx.x, g, g & 1u, cpi, a.pop[g & 1u], sm);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->gens_run = g;
+}
+
+// ------------------------------------------------------------------------
+// Small kernels
+// ------------------------------------------------------------------------
+__global__ void eval_stats_kernel(ChainDev ch, const uint64_t* bits, int64_t* st_out, double* f_out)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint32_t* s_chain = (uint32_t*)smem;
+    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
+    stage_chain(s_chain, ch, mbar);
+    if (threadIdx.x == 0) {
+        Stats st{};
+        const double f = eval_walk(ch, s_chain, s_chain + ch.p_words, [&](uint32_t w) { return bits[w]; }, &st);
+        st_out[0] = st.k; st_out[1] = st.V; st_out[2] = (int64_t)st.S1; st_out[3] = (int64_t)st.S2; st_out[4] = (int64_t)st.OV;
+        *f_out = f;
+    }
+}
+
+__global__ void selftest_philox_kernel(const uint32_t* in, uint32_t n, uint32_t* out)
+{
+    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= n) return;
+    const uint32_t* v = in + 6 * t;
+    const uint4 r = philox10(make_uint4(v[0], v[1], v[2], v[3]), v[4], v[5]);
+    out[4 * t] = r.x; out[4 * t + 1] = r.y; out[4 * t + 2] = r.z; out[4 * t + 3] = r.w;
+}
+
+__global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
+{
+    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < n) out[t] = dexp_dev(in[t]);
+}
+
+// ------------------------------------------------------------------------
+// Launchers
+// ------------------------------------------------------------------------
+static size_t eval_smem(const ChainDev& ch)
+{
+    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
+}
+
+cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out, cudaStream_t st,
+                              int num_sms, uint64_t* launches)
+{
+    if (n_cand == 0) return cudaSuccess;
+    const size_t sm = eval_smem(ch);
+    cudaError_t e = cudaFuncSetAttribute(eval_batch_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, eval_batch_kernel, kEvalWarps * 32, sm);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+    const uint64_t tiles = (n_cand + 31) / 32;
+    uint64_t grid = (uint64_t)per_sm * num_sms;
+    const uint64_t need = (tiles + kEvalWarps - 1) / kEvalWarps;
+    if (grid > need) grid = need;
+    eval_batch_kernel<<<(unsigned)grid, kEvalWarps * 32, sm, st>>>(ch, bits, n_cand, out);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+size_t ga_smem_bytes(const GaArgs& a) { return smem_layout(a, nullptr, nullptr); }
+
+template <int WT>
+static void* ga_fn()
+{
+    return (void*)ga_kernel<WT>;
+}
+
+static void* ga_pick(uint32_t W)
+{
+    if (W <= 1) return ga_fn<1>();
+    if (W <= 2) return ga_fn<2>();
+    if (W <= 4) return ga_fn<4>();
+    if (W <= 8) return ga_fn<8>();
+    if (W <= 16) return ga_fn<16>();
+    return ga_fn<64>();
+}
+
+int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err)
+{
+    void* fn = ga_pick(a.ch.W);
+    const size_t sm = ga_smem_bytes(a);
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    int per_sm = 0;
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kBlock, sm);
+    if (err) *err = e;
+    if (e != cudaSuccess || per_sm < 1) return 0;
+    return per_sm * num_sms;
+}
+
+cudaError_t launch_ga(const GaArgs& a, cudaStream_t st, int num_sms, uint64_t* launches)
+{
+    cudaError_t e;
+    const int grid = ga_grid(a, num_sms, &e);
+    if (e != cudaSuccess) return e;
+    if (grid < (int)a.I) return cudaErrorInvalidConfiguration;
+    void* fn = ga_pick(a.ch.W);
+    GaArgs copy = a;
+    void* args[] = {&copy};
+    e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, ga_smem_bytes(a), st);
+    if (launches) ++*launches;
+    return e;
+}
+
+cudaError_t launch_eval_stats(const ChainDev& ch, const uint64_t* bits, int64_t* stats_out, double* f_out,
+                              cudaStream_t st)
+{
+    const size_t sm = (size_t)(ch.p_words + ch.o_words) * 4 + 16;
+    cudaError_t e = cudaFuncSetAttribute(eval_stats_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+    eval_stats_kernel<<<1, 32, sm, st>>>(ch, bits, stats_out, f_out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_selftest_philox(const uint32_t* in, uint32_t n, uint32_t* out, cudaStream_t st)
+{
+    if (n == 0) return cudaSuccess;
+    selftest_philox_kernel<<<(n + 127) / 128, 128, 0, st>>>(in, n, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_selftest_dexp(const double* in, uint32_t n, double* out, cudaStream_t st)
+{
+    if (n == 0) return cudaSuccess;
+    selftest_dexp_kernel<<<(n + 127) / 128, 128, 0, st>>>(in, n, out);
+    return cudaGetLastError();
+}
+
+}  // namespace splitga

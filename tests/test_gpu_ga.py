@@ -1,0 +1,143 @@
+"""GPU parity of split_ga_run (a1, a3-a9) against the oracle GA: the best
+record, counters and the whole population (every row and every fitness bit)
+after G generations must be identical.  All calls go through the C ABI."""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ORACLE_KEYS = ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max",
+               "front_skip", "stall_generations", "n_islands", "migration_interval", "n_migrants")
+
+
+@pytest.fixture(scope="module")
+def S():
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA not available on a GPU test run")
+    from paper_conf_icpp_luoyww0023_b200 import split
+    return split
+
+
+def _fbits(x):
+    return np.asarray(x, np.float64).view(np.uint64)
+
+
+def run_both(S, lat, ovh, G, seed, check_pop=True, **kw):
+    kw.setdefault("islands_per_device", kw.get("n_islands", 1))
+    h = S.SplitGA(lat, ovh, **kw)
+    r = h.run(G, seed)
+    okw = {k: v for k, v in kw.items() if k in ORACLE_KEYS}
+    o = oracle.ga_run(lat, ovh, G, seed, want_population=check_pop, **okw)
+    assert r["fitness"] == o["fitness"] or (math.isinf(r["fitness"]) and math.isinf(o["fitness"]))
+    assert np.array_equal(r["bits"], o["bits"])
+    for key in ("k", "var_num", "s1", "s2", "generation_found", "generations_run", "evaluations"):
+        assert r[key] == o[key], (key, r[key], o[key])
+    assert r["overhead_ns"] == o["overhead"]
+    if check_pop:
+        for i in range(kw.get("n_islands", 1)):
+            bits, fit = h.population(i)
+            assert np.array_equal(bits, o["population"][i]), f"island {i} rows differ"
+            assert np.array_equal(_fbits(fit), _fbits(o["fitness_all"][i])), f"island {i} fitness differ"
+    stats = h.last_run_stats()
+    h.close()
+    return r, o, stats
+
+
+@pytest.mark.parametrize("seed", [1, 42, 20230807])
+@pytest.mark.parametrize("G", [0, 1, 2, 7, 50])
+def test_c1_trajectory(S, seed, G):
+    lat, ovh = wl.c1_chain()
+    run_both(S, lat, ovh, G, seed, pop_size=256, n_elite=4, k_min=2, k_max=12)
+
+
+@pytest.mark.parametrize("k", list(range(2, 13)))
+def test_c1_fixed_k_reaches_brute_force(S, k):
+    lat, ovh = wl.c1_chain(overhead="const")
+    r, o, _ = run_both(S, lat, ovh, 50, 42, pop_size=256, n_elite=4, k_min=k, k_max=k)
+    b = oracle.brute(lat, ovh, k, k)
+    assert r["fitness"] == b["fitness"] and int(r["bits"][0]) == b["bits"]
+
+
+@pytest.mark.parametrize("name,N,E,G", [("resnet50_175", 4096, 82, 12), ("vgg16", 2048, 40, 20),
+                                        ("bert_base", 2048, 40, 8), ("synthetic_1024", 1024, 20, 6),
+                                        ("mobilenetv2", 8192, 1024, 6), ("gpt2", 256, 6, 4)])
+def test_model_chains(S, name, N, E, G):
+    lat, ovh = wl.chain(name)
+    run_both(S, lat, ovh, G, 7, pop_size=N, n_elite=E, k_min=2, k_max=min(32, len(lat)))
+
+
+def test_general_select_path_exercised(S):
+    # a large random-ish population makes many children beat the worst elite early on,
+    # forcing the radix top-E path; later generations use the candidate merge
+    lat, ovh = wl.chain("resnet50_175")
+    r, o, st = run_both(S, lat, ovh, 15, 3, pop_size=20000, n_elite=1024, k_min=2, k_max=32)
+    assert st["general_selects"] >= 2 and st["fast_selects"] >= 1
+
+
+@pytest.mark.parametrize("kw", [
+    dict(pop_size=100, n_elite=0),
+    dict(pop_size=64, n_elite=64),
+    dict(pop_size=130, n_elite=2, tournament_size=1),
+    dict(pop_size=130, n_elite=2, tournament_size=32),
+    dict(pop_size=128, n_elite=8, p_crossover=0.0, p_mutation=0.0, k_min=1, k_max=105),
+    dict(pop_size=128, n_elite=8, p_crossover=1.0, p_mutation=1.0),
+    dict(pop_size=128, n_elite=8, k_min=5, k_max=5, front_skip=60),
+    dict(pop_size=128, n_elite=8, k_min=1, k_max=3),
+])
+def test_edge_parameters(S, kw):
+    lat, ovh = wl.chain("mobilenetv2")
+    base = dict(k_min=2, k_max=32)
+    base.update(kw)
+    run_both(S, lat, ovh, 9, 11, **base)
+
+
+def test_stall_termination(S):
+    lat, ovh = wl.c1_chain()
+    r, o, _ = run_both(S, lat, ovh, 500, 1, pop_size=256, n_elite=4, k_min=2, k_max=12, stall_generations=15)
+    assert r["generations_run"] < 500
+
+
+def test_zero_chain_ties(S):
+    lat, ovh = wl.c1_chain(overhead="ties")
+    run_both(S, lat, ovh, 30, 5, pop_size=256, n_elite=4, k_min=2, k_max=12)
+
+
+@pytest.mark.parametrize("M,stall", [(3, 0), (0, 0), (4, 8)])
+def test_local_islands_with_migration(S, M, stall):
+    lat, ovh = wl.chain("resnet50_175")
+    run_both(S, lat, ovh, 13, 77, pop_size=128, n_elite=4, k_min=2, k_max=16, n_islands=4,
+             migration_interval=M, n_migrants=4 if M else 0, stall_generations=stall)
+
+
+def test_islands_eight_large_migrants(S):
+    lat, ovh = wl.chain("bert_base")
+    run_both(S, lat, ovh, 10, 9, pop_size=512, n_elite=16, k_min=2, k_max=32, n_islands=8,
+             migration_interval=2, n_migrants=64)
+
+
+def test_c2_full_size_first_generations(S):
+    """C2 at the size bench.py runs (n = 175, N = 65,536, E = 1024): the first
+    generations are compared bit for bit with the oracle."""
+    lat, ovh = wl.chain("resnet50_175")
+    run_both(S, lat, ovh, 4, 20230807, pop_size=65536, n_elite=1024, k_min=2, k_max=32)
+
+
+def test_c2_full_run_invariants(S):
+    lat, ovh = wl.chain("resnet50_175")
+    h = S.SplitGA(lat, ovh, pop_size=65536, n_elite=1024, k_min=2, k_max=32)
+    r = h.run(500, 1)
+    bits, fit = h.population(0)
+    h.close()
+    assert r["generations_run"] == 500 and r["evaluations"] == 65536 + 500 * 64512
+    assert np.all(np.diff(fit[:1024]) <= 0)          # elites in rank order
+    assert r["fitness"] >= fit.max()
+    # the reported best re-evaluates to itself on the oracle
+    s = oracle.fitness(lat, ovh, r["bits"], 2, 32)
+    assert s["fitness"] == r["fitness"] and s["var_num"] == r["var_num"] and s["k"] == r["k"]
+    assert r["expected_wait_ns"] == pytest.approx(s["s2"] / (2 * s["s1"]))
