@@ -7,6 +7,7 @@
 #include <nccl.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -164,6 +165,8 @@ struct split_ga_t {
     uint64_t* d_bits1;
     uint64_t* d_recpack;   // [I_total][W + 2]
     cudaEvent_t ev[4];
+    unsigned long long* d_trace;   // SPLIT_TRACE=<csv path>: phase timestamps of the first RUN segment
+    uint32_t trace_gens;
     // eval_batch_host staging
     uint64_t* d_hbits[2];
     double* d_hfit[2];
@@ -371,22 +374,30 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
         delete h;
         return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s", cudaGetErrorString(ge));
     }
-    h->cpi = (uint32_t)h->grid / a.I;
+    if (h->grid < 2 * (int)a.I) {
+        free_all(h);
+        delete h;
+        return fail(SPLIT_E_INVAL, "grid %d too small for %u islands", h->grid, a.I);
+    }
+    h->cpi = (uint32_t)(h->grid - (int)a.I) / a.I;
     const size_t IN = (size_t)a.I * a.N;
     for (int b = 0; b < 2; ++b) {
         TRY(dalloc(h, &a.pop[b], IN * h->W));
         TRY(dalloc(h, &a.fit[b], IN));
+    }
+    for (int b = 0; b < 3; ++b) {
         TRY(dalloc(h, &a.cand_key[b], IN));
         TRY(dalloc(h, &a.cand_idx[b], IN));
     }
-    TRY(dalloc(h, &a.cand_cnt, 2 * (size_t)a.I));
+    TRY(dalloc(h, &a.cand_cnt, 3 * (size_t)a.I));
     TRY(dalloc(h, &a.sel_key, (size_t)a.I * kMaxElite));
     TRY(dalloc(h, &a.sel_idx, (size_t)a.I * kMaxElite));
     TRY(dalloc(h, &a.sel_cnt, a.I));
-    TRY(dalloc(h, &a.tau, a.I));
+    TRY(dalloc(h, &a.tau, 2 * (size_t)a.I));
     TRY(dalloc(h, &a.ghist, 3 * (size_t)a.I * 256));
     TRY(dalloc(h, &a.part_f, 2 * (size_t)a.I * h->cpi));
     TRY(dalloc(h, &a.part_idx, 2 * (size_t)a.I * h->cpi));
+    TRY(dalloc(h, &a.part_bits, 2 * (size_t)a.I * h->cpi * h->W));
     TRY(dalloc(h, &a.rec_f, a.I));
     TRY(dalloc(h, &a.rec_bits, (size_t)a.I * h->W));
     TRY(dalloc(h, &a.rec_gen, a.I));
@@ -398,6 +409,10 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     TRY(dalloc(h, &h->d_statf, 1));
     TRY(dalloc(h, &h->d_bits1, h->W));
     TRY(dalloc(h, &h->d_recpack, (size_t)a.I_total * (h->W + 2)));
+    if (getenv("SPLIT_TRACE")) {
+        h->trace_gens = 64;
+        TRY(dalloc(h, &h->d_trace, (size_t)h->trace_gens * 8));
+    }
     for (int i = 0; i < 4; ++i) {
         cudaError_t e = cudaEventCreate(&h->ev[i]);
         if (e != cudaSuccess) TRY(fail(SPLIT_E_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
@@ -473,6 +488,8 @@ static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
 {
     GaArgs a = h->ga;
     a.mode = mode;
+    a.trace = (mode == MODE_RUN) ? h->d_trace : nullptr;
+    a.trace_gens = h->trace_gens;
     a.g_begin = g0;
     a.g_end = g1;
     cudaError_t e = launch_ga(a, h->stream, h->num_sms, &h->stats.launches);
@@ -555,9 +572,10 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     a.stall_in_kernel = single ? 1u : 0u;
     h->stats = split_run_stats{};
     CU(cudaMemsetAsync(a.rec_valid, 0, a.I * 4, h->stream));
-    CU(cudaMemsetAsync(a.cand_cnt, 0, 2 * a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.cand_cnt, 0, 3 * a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.sel_cnt, 0, a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.ghist, 0, 3 * a.I * 256 * 4, h->stream));
+    CU(cudaMemsetAsync(a.tau, 0xFF, 2 * a.I * 8, h->stream));
     CU(cudaEventRecord(h->ev[0], h->stream));
     int rc = run_kernel(h, MODE_INIT, 0, 0);
     if (rc) return rc;
@@ -641,6 +659,19 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     best_out->evaluations = (uint64_t)a.I * ((uint64_t)a.N + (uint64_t)gens_run * (a.N - a.E));
     h->last_gen = gens_run;
     h->have_pop = true;
+    if (h->d_trace) {
+        std::vector<unsigned long long> tr((size_t)h->trace_gens * 8);
+        CU(cudaMemcpy(tr.data(), h->d_trace, tr.size() * 8, cudaMemcpyDeviceToHost));
+        if (FILE* f = fopen(getenv("SPLIT_TRACE"), "w")) {
+            fprintf(f, "gen,lead_start,lead_record,lead_sort,lead_end,work_start,work_end,lead_sync,work_sync\n");
+            for (uint32_t g = 0; g < h->trace_gens; ++g) {
+                fprintf(f, "%u", g);
+                for (int j = 0; j < 8; ++j) fprintf(f, ",%llu", tr[(size_t)g * 8 + j]);
+                fprintf(f, "\n");
+            }
+            fclose(f);
+        }
+    }
     if (fchk != best.f) return fail(SPLIT_E_STATE, "best record fitness mismatch (internal)");
     return SPLIT_OK;
 }

@@ -50,16 +50,17 @@ struct GaArgs {
     uint32_t sort_cap;                 // power of two, entries the leader can sort in smem
     uint64_t* pop[2];                  // [I][N][W]
     double* fit[2];                    // [I][N]
-    uint64_t* cand_key[2];             // [I][N]   candidates of generation g (parity g&1)
-    uint32_t* cand_idx[2];
-    uint32_t* cand_cnt;                // [2][I]
+    uint64_t* cand_key[3];             // [I][N]   candidates of generation g (list g%3)
+    uint32_t* cand_idx[3];
+    uint32_t* cand_cnt;                // [3][I]
     uint64_t* sel_key;                 // [I][kMaxElite] general-select / elite output
     uint32_t* sel_idx;
     uint32_t* sel_cnt;                 // [I]
-    uint64_t* tau;                     // [I] key of the worst elite of the current generation
+    uint64_t* tau;                     // [2][I] key of the worst elite of generation g (parity g&1)
     uint32_t* ghist;                   // [3][I][256]
     double* part_f;                    // [2][I][cpi] per-CTA best child
     uint32_t* part_idx;
+    uint64_t* part_bits;               // [2][I][cpi][W] bits of each per-CTA best
     double* rec_f;                     // [I] island records
     uint64_t* rec_bits;                // [I][W]
     uint32_t* rec_gen;                 // [I]
@@ -67,6 +68,8 @@ struct GaArgs {
     uint64_t* mig_bits;                // [I_total][K][W]
     double* mig_f;                     // [I_total][K]
     Ctl* ctl;
+    unsigned long long* trace;         // optional phase timestamps (SPLIT_TRACE), [trace_gens][8]
+    uint32_t trace_gens;
 };
 
 // Launchers (split_kernels.cu).  Return cudaError_t of the launch.

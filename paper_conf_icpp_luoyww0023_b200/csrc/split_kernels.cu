@@ -106,6 +106,21 @@ __device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, uint32
     return -__dadd_rn(dexp_dev(__dsub_rn(x, 1.0)), dexp_dev(__dsub_rn(y, 1.0)));
 }
 
+__device__ __forceinline__ unsigned long long gtimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// phase timestamps (SPLIT_TRACE): leader CTA 0 slots 0-3, last worker CTA 4-5,
+// after the generation barrier 6 (CTA 0) and 7 (last CTA)
+__device__ __forceinline__ void trace_mark(const GaArgs& a, uint32_t g, uint32_t slot)
+{
+    if (!a.trace || threadIdx.x != 0 || blockIdx.x != 0) return;
+    const uint32_t gi = g - a.g_begin;
+    if (gi < a.trace_gens) a.trace[gi * 8 + slot] = gtimer();
+}
+
 // order-preserving u64 key of a fitness (larger f -> larger key)
 __device__ __forceinline__ uint64_t fkey(double f)
 {
@@ -247,6 +262,95 @@ __global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_kernel(ChainDev ch
         if (lane < rows) {
             const uint64_t* my = tile + lane * pitch;
             const double f = eval_walk(ch, sP, sO, [&](uint32_t w) { return my[w]; }, nullptr);
+            __stcs(out + row0 + lane, f);
+        }
+        __syncwarp();
+    }
+}
+
+// K1 for W <= 16 (n_ops <= 1025): W is a compile-time constant, rows are
+// handled as 2W 32-bit half-words and each lane keeps a bitmask of its
+// non-empty half-words, so the walk takes exactly one iteration per cut
+// (no per-word loop whose trip count diverges across the warp).
+template <int W>
+__global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
+                                                                       uint64_t n_cand, double* __restrict__ out)
+{
+    constexpr uint32_t H = 2 * W;          // 32-bit halves per row
+    constexpr uint32_t PITCH = H + 1;      // odd pitch: lanes read distinct banks
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint32_t* s_chain = (uint32_t*)smem;
+    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
+    uint32_t* s_tiles = (uint32_t*)(mbar + 2);
+    stage_chain(s_chain, ch, mbar);
+    const uint32_t* sP = s_chain;
+    const uint32_t* sO = s_chain + ch.p_words;
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint32_t* tile = s_tiles + warp * 32u * PITCH;
+    // valid bits: positions [0, n-2] -> halves [0, qfull) full, half qfull partial
+    const uint32_t npos = ch.n - 1, qfull = npos >> 5;
+    const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
+    const uint64_t n_tiles = (n_cand + 31) / 32;
+    const uint64_t nw = (uint64_t)gridDim.x * kEvalWarps;
+    for (uint64_t t = (uint64_t)blockIdx.x * kEvalWarps + warp; t < n_tiles; t += nw) {
+        const uint64_t row0 = t * 32;
+        const uint32_t rows = (uint32_t)((n_cand - row0) < 32 ? (n_cand - row0) : 32);
+        if (rows == 32) {
+            const uint4* src4 = (const uint4*)(bits + row0 * W);   // 256*W bytes, 16-byte aligned
+#pragma unroll
+            for (uint32_t it = 0; it < (16 * W + 31) / 32; ++it) {
+                const uint32_t j = lane + 32 * it;
+                if (j < 16 * W) {
+                    const uint4 v = __ldcs(src4 + j);
+                    const uint32_t e = 4 * j;       // first half-word of the chunk; e and H are even
+                    const uint32_t r = e / H, c = e % H;
+                    uint32_t* d = tile + r * PITCH + c;
+                    d[0] = v.x; d[1] = v.y;
+                    if (c + 2 < H) { d[2] = v.z; d[3] = v.w; }
+                    else { d[PITCH - c] = v.z; d[PITCH - c + 1] = v.w; }   // c + 2 == H: row r+1, halves 0-1
+                }
+            }
+        } else {
+            const uint32_t* src = (const uint32_t*)(bits + row0 * W);
+            for (uint32_t e = lane; e < rows * H; e += 32) tile[(e / H) * PITCH + (e % H)] = __ldcs(src + e);
+        }
+        __syncwarp();
+        if (lane < rows) {
+            const uint32_t* my = tile + lane * PITCH;
+            uint32_t cuts = 0, occ = 0;
+#pragma unroll
+            for (uint32_t q = 0; q < H; ++q) {
+                uint32_t v = my[q];
+                v &= (q < qfull) ? ~0u : (q == qfull ? lastm : 0u);
+                cuts += __popc(v);
+                occ |= (v != 0u ? 1u : 0u) << q;
+            }
+            const uint32_t k = cuts + 1;
+            double f = -CUDART_INF;
+            if (k >= ch.k_min && k <= ch.k_max) {
+                uint32_t startP = 0, prev_o = 0, OV = 0, v = 0, q = 0;
+                uint64_t S2 = 0;
+                for (uint32_t j = 0; j < cuts; ++j) {
+                    if (v == 0u) {
+                        q = __ffs(occ) - 1;
+                        occ &= occ - 1;
+                        v = my[q] & ((q < qfull) ? ~0u : lastm);
+                    }
+                    const uint32_t p = 32u * q + (uint32_t)(__ffs(v) - 1);
+                    v &= v - 1;
+                    const uint32_t Pp = sP[p + 1];
+                    const uint32_t tj = Pp - startP + prev_o;
+                    S2 += (uint64_t)tj * tj;
+                    prev_o = sO[p];
+                    OV += prev_o;
+                    startP = Pp;
+                }
+                const uint32_t tl = ch.T - startP + prev_o;
+                S2 += (uint64_t)tl * tl;
+                const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
+                const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+                f = eq2(k, V, OV, ch.T);
+            }
             __stcs(out + row0 + lane, f);
         }
         __syncwarp();
@@ -406,6 +510,90 @@ __device__ BestRef block_best(BestRef v, const uint64_t* base, uint32_t W, BestR
     return r;
 }
 
+// A candidate best record carried in registers: (f, index, bits).  Ties on f
+// are broken on the bits themselves (R10), so no reduction re-reads rows.
+template <int WT>
+struct BestRow {
+    double f;
+    uint32_t idx;
+    uint32_t pad;
+    Row<WT> r;
+};
+
+template <int WT>
+__device__ __forceinline__ bool better_row(const BestRow<WT>& a, const BestRow<WT>& b, uint32_t W)
+{
+    if (a.idx == NONE) return false;
+    if (b.idx == NONE) return true;
+    if (a.f != b.f) return a.f > b.f;
+    bool less = false, decided = false;
+#pragma unroll
+    for (int w = WT - 1; w >= 0; --w)
+        if (w < (int)W && !decided && a.r.w[w] != b.r.w[w]) { less = a.r.w[w] < b.r.w[w]; decided = true; }
+    return less;
+}
+
+template <int WT>
+__device__ __forceinline__ BestRow<WT> shfl_down_row(const BestRow<WT>& v, int off, uint32_t W)
+{
+    BestRow<WT> o;
+    o.f = __shfl_down_sync(0xFFFFFFFFu, v.f, off);
+    o.idx = __shfl_down_sync(0xFFFFFFFFu, v.idx, off);
+    o.pad = 0;
+#pragma unroll
+    for (int i = 0; i < WT; ++i) o.r.w[i] = (i < (int)W) ? __shfl_down_sync(0xFFFFFFFFu, v.r.w[i], off) : 0ull;
+    return o;
+}
+
+// block-wide best over BestRow candidates; all threads call; scratch: 33 entries
+template <int WT>
+__device__ BestRow<WT> block_best_row(BestRow<WT> v, uint32_t W, BestRow<WT>* scratch)
+{
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+#pragma unroll
+    for (int off = 16; off; off >>= 1) {
+        const BestRow<WT> o = shfl_down_row(v, off, W);
+        if (lane + off < 32 && better_row(o, v, W)) v = o;
+    }
+    if (lane == 0) scratch[warp] = v;
+    __syncthreads();
+    if (warp == 0) {
+        if (lane < nwarps) v = scratch[lane];
+        else { v.f = -CUDART_INF; v.idx = NONE; }
+#pragma unroll
+        for (int off = 16; off; off >>= 1) {
+            const BestRow<WT> o = shfl_down_row(v, off, W);
+            if (lane + off < 32 && better_row(o, v, W)) v = o;
+        }
+        if (lane == 0) scratch[32] = v;
+    }
+    __syncthreads();
+    const BestRow<WT> r = scratch[32];
+    __syncthreads();
+    return r;
+}
+
+template <int WT>
+__device__ __forceinline__ void track_row(BestRow<WT>& b, double f, uint32_t idx, const Row<WT>& r, uint32_t W)
+{
+    BestRow<WT> c;
+    c.f = f;
+    c.idx = idx;
+    c.pad = 0;
+    c.r = r;
+    if (better_row(c, b, W)) b = c;
+}
+
+template <int WT>
+__device__ __forceinline__ void write_partial(const GaArgs& a, size_t slot, const BestRow<WT>& b, uint32_t W)
+{
+    a.part_f[slot] = b.f;
+    a.part_idx[slot] = b.idx;
+#pragma unroll
+    for (int i = 0; i < WT; ++i)
+        if (i < (int)W) a.part_bits[slot * W + i] = b.r.w[i];
+}
+
 // composite ranking order (key desc, idx asc)
 __device__ __forceinline__ bool comp_gt(uint64_t ka, uint32_t ia, uint64_t kb, uint32_t ib)
 {
@@ -479,9 +667,14 @@ struct Smem {
     uint64_t* skey;       // [sort_cap]
     uint32_t* sidx;       // [sort_cap]
     uint64_t* ekey;       // [kMaxElite]
+    uint64_t* okey;       // [kMaxElite] merged elites (fast path)
+    uint32_t* oidx;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
+
+// register-row width (template WT) used for a row of W words
+__host__ __device__ inline uint32_t wt_of(uint32_t W) { return W <= 1 ? 1 : W <= 2 ? 2 : W <= 4 ? 4 : W <= 8 ? 8 : W <= 16 ? 16 : 64; }
 
 __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Smem* s)
 {
@@ -492,10 +685,12 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take(16); if (s) s->mbar = (uint64_t*)p;
     p = take((size_t)a.I * 256 * 4); if (s) s->hist = (uint32_t*)p;
     p = take((size_t)a.I * sizeof(SelState)); if (s) s->sel = (SelState*)p;
-    p = take(33 * sizeof(BestRef)); if (s) s->scratch = (BestRef*)p;
+    p = take(33 * (16 + 8 * (size_t)wt_of(a.ch.W))); if (s) s->scratch = (BestRef*)p;   // 33 BestRow<WT>
     p = take((size_t)a.sort_cap * 8); if (s) s->skey = (uint64_t*)p;
     p = take((size_t)a.sort_cap * 4); if (s) s->sidx = (uint32_t*)p;
     p = take((size_t)kMaxElite * 8); if (s) s->ekey = (uint64_t*)p;
+    p = take((size_t)kMaxElite * 8); if (s) s->okey = (uint64_t*)p;
+    p = take((size_t)kMaxElite * 4); if (s) s->oidx = (uint32_t*)p;
     return off;
 }
 
@@ -660,32 +855,46 @@ __device__ void leader_sort_selected(const GaArgs& a, uint32_t i, uint32_t Ksel,
 }
 
 // Leader CTA: record update of island i from the per-CTA partial bests of
-// generation g (rows in pop_g), and the single-island stall rule (R11).
-__device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t parity, uint32_t cpi,
-                              const uint64_t* pop_g, const Smem& sm)
+// generation g (f, index and bits, in part_*), and the single-island stall
+// rule (R11).
+template <int WT>
+__device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t parity, uint32_t cpi, const Smem& sm)
 {
     const uint32_t W = a.ch.W;
-    const uint64_t* base = pop_g + (size_t)i * a.N * W;
-    BestRef v{-CUDART_INF, NONE};
-    const double* pf = a.part_f + ((size_t)parity * a.I + i) * cpi;
-    const uint32_t* pi = a.part_idx + ((size_t)parity * a.I + i) * cpi;
+    BestRow<WT> v;
+    v.f = -CUDART_INF;
+    v.idx = NONE;
+    const size_t base = ((size_t)parity * a.I + i) * cpi;
     for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x) {
-        const BestRef o{pf[j], pi[j]};
-        if (better_rec(o.f, o.idx, v.f, v.idx, base, W)) v = o;
+        BestRow<WT> o;
+        o.f = __ldcg(a.part_f + base + j);
+        o.idx = __ldcg(a.part_idx + base + j);
+#pragma unroll
+        for (int w = 0; w < WT; ++w) o.r.w[w] = (w < (int)W) ? __ldcg(a.part_bits + (base + j) * W + w) : 0ull;
+        if (better_row(o, v, W)) v = o;
     }
-    v = block_best(v, base, W, sm.scratch);
+    v = block_best_row(v, W, (BestRow<WT>*)sm.scratch);
     if (threadIdx.x == 0) {
         bool upd = false;
         if (v.idx != NONE) {
             if (!a.rec_valid[i]) upd = true;
             else if (v.f != a.rec_f[i]) upd = v.f > a.rec_f[i];
-            else upd = rows_less(base + (size_t)v.idx * W, a.rec_bits + (size_t)i * W, W);
+            else {
+                BestRow<WT> rec;
+                rec.f = v.f;
+                rec.idx = 0;
+#pragma unroll
+                for (int w = 0; w < WT; ++w) rec.r.w[w] = (w < (int)W) ? a.rec_bits[(size_t)i * W + w] : 0ull;
+                upd = better_row(v, rec, W);
+            }
         }
         if (upd) {
             a.rec_f[i] = v.f;
             a.rec_gen[i] = g;
             a.rec_valid[i] = 1;
-            for (uint32_t w = 0; w < W; ++w) a.rec_bits[(size_t)i * W + w] = base[(size_t)v.idx * W + w];
+#pragma unroll
+            for (int w = 0; w < WT; ++w)
+                if (w < (int)W) a.rec_bits[(size_t)i * W + w] = v.r.w[w];
         }
         if (a.stall_in_kernel && i == 0) {
             Ctl* c = a.ctl;
@@ -760,72 +969,151 @@ __device__ __forceinline__ void init_row(const GaArgs& a, Row<WT>& row, uint32_t
     }
 }
 
-// per-thread running best child, (f desc, bits asc); rows already in pop_n
+// One child per thread.  The two children of a pair (c0 = E + 2q, c1 = c0 + 1)
+// sit in adjacent lanes and swap their tournament winners with one shuffle;
+// each lane then builds only its own child (R8, R18).
 template <int WT>
-__device__ __forceinline__ void track_best(BestRef& b, double f, uint32_t idx, const Row<WT>& r,
-                                           const uint64_t* pop_island, uint32_t W)
+__device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl, uint32_t cpi,
+                                               const uint64_t* popc, const double* fitc, uint64_t* popn,
+                                               double* fitn, const uint32_t* sP, const uint32_t* sO, uint64_t tau,
+                                               uint32_t* ccnt, uint64_t* ckey, uint32_t* cidx, BestRow<WT>& best)
 {
-    if (b.idx == NONE || f > b.f) { b.f = f; b.idx = idx; return; }
-    if (f < b.f) return;
-    const uint64_t* o = pop_island + (size_t)b.idx * W;
-    for (int w = (int)W - 1; w >= 0; --w) {
-        uint64_t mine = 0;
+    const ChainDev& ch = a.ch;
+    const uint32_t W = ch.W, N = a.N, E = a.E;
+    const uint32_t nchild = N - E;
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t stride = cpi * blockDim.x;
+    for (uint32_t base = wl * blockDim.x + (threadIdx.x & ~31u); base < nchild; base += stride) {
+        const uint32_t t = base + lane;
+        const bool valid = t < nchild;
+        const uint32_t h = t & 1u;
+        const uint32_t slot = E + t;
+        const uint32_t gid = (a.island_base + i) * N + slot;
+        const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc) : 0u;     // a4
+        const uint32_t other = __shfl_xor_sync(0xFFFFFFFFu, mine, 1);
+        if (!valid) continue;
+        // first parent (positions < x) = own winner; second = the partner's
+        Row<WT> A, B;
+        row_load(A, popc + (size_t)mine * W, W);
+        row_load(B, popc + (size_t)other * W, W);
+        const uint4 rx = philox10(make_uint4(gid - h, g, TAG_XOVER, 0), a.key0, a.key1);   // a5
+        if ((uint64_t)rx.x < a.thr_c && ch.n >= 3) {
+            const uint32_t x = 1 + below(rx.y, ch.n - 2);
 #pragma unroll
-        for (int i = 0; i < WT; ++i)
-            if (i == w) mine = r.w[i];
-        if (mine != o[w]) {
-            if (mine < o[w]) { b.f = f; b.idx = idx; }
-            return;
+            for (int w = 0; w < WT; ++w) {
+                const uint32_t lo = 64u * w;
+                const uint64_t m = (x >= lo + 64) ? ~0ull : (x <= lo ? 0ull : ((1ull << (x - lo)) - 1));
+                A.w[w] = (A.w[w] & m) | (B.w[w] & ~m);
+            }
         }
+        const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);     // a6
+        if ((uint64_t)rm.x < a.thr_m) row_xor_bit(A, below(rm.y, ch.n - 1));
+        repair(a, A, gid, g);                                                              // a7
+        const double f = eval_regs(ch, sP, sO, A, nullptr);                               // a2
+        row_store(A, popn + (size_t)slot * W, W);
+        fitn[slot] = f;
+        append_if(fkey(f) > tau, ccnt, ckey, cidx, fkey(f), slot);
+        track_row(best, f, slot, A, W);
     }
 }
 
+// Leader CTA of island i in the phase of generation g: record + stall of
+// generation g (a8), elites of generation g into slots 0..E-1 of g+1 (a3),
+// worst-elite key tau of generation g, reset of the candidate list that the
+// breed of the NEXT phase appends to.
 template <int WT>
-__device__ __forceinline__ void breed_pair(const GaArgs& a, uint32_t i, uint32_t q, uint32_t g, const uint64_t* popc,
-                                           const double* fitc, uint64_t* popn, double* fitn, const uint32_t* sP,
-                                           const uint32_t* sO, uint64_t tau, uint32_t* ccnt, uint64_t* ckey,
-                                           uint32_t* cidx, BestRef& best)
+__device__ void leader_phase(const GaArgs& a, uint32_t i, uint32_t g, bool general, uint32_t cpi, const Smem& sm)
 {
-    const ChainDev& ch = a.ch;
-    const uint32_t W = ch.W, N = a.N;
-    const uint32_t c0 = a.E + 2 * q;
-    const uint32_t gid0 = (a.island_base + i) * N + c0;
-    const uint32_t pa = tournament<WT>(a, gid0, g, fitc);
-    const uint32_t pb = tournament<WT>(a, gid0 + 1, g, fitc);
-    Row<WT> A, B;
-    row_load(A, popc + (size_t)pa * W, W);
-    row_load(B, popc + (size_t)pb * W, W);
-    const uint4 rx = philox10(make_uint4(gid0, g, TAG_XOVER, 0), a.key0, a.key1);
-    if ((uint64_t)rx.x < a.thr_c && ch.n >= 3) {
-        const uint32_t x = 1 + below(rx.y, ch.n - 2);   // positions < x from the first parent
-#pragma unroll
-        for (int w = 0; w < WT; ++w) {
-            const uint32_t lo = 64u * w;
-            const uint64_t m = (x >= lo + 64) ? ~0ull : (x <= lo ? 0ull : ((1ull << (x - lo)) - 1));
-            const uint64_t a0 = A.w[w], b0 = B.w[w];
-            A.w[w] = (a0 & m) | (b0 & ~m);
-            B.w[w] = (b0 & m) | (a0 & ~m);
+    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I;
+    const uint32_t cur = g & 1u, nxt = cur ^ 1u;
+    const uint32_t Lc = g % 3u, Lr = (g + 2u) % 3u;
+    trace_mark(a, g, 0);
+    leader_record<WT>(a, i, g, cur, cpi, sm);
+    trace_mark(a, g, 1);
+    const uint64_t* popc = a.pop[cur] + (size_t)i * N * W;
+    const double* fitc = a.fit[cur] + (size_t)i * N;
+    if (E > 0) {
+        if (general) {
+            leader_sort_selected(a, i, E, false, sm);
+        } else {
+            // previous elites (slots 0..E-1, ranked) merged with the candidates that
+            // beat the worst of them; the candidate list is a superset (lagged tau)
+            for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) sm.ekey[r] = fkey(__ldcg(fitc + r));
+            __syncthreads();
+            const uint64_t thr = sm.ekey[E - 1];
+            const uint32_t C0 = __ldcg(&a.cand_cnt[Lc * I + i]);
+            const uint64_t* ck = a.cand_key[Lc] + (size_t)i * N;
+            const uint32_t* cx = a.cand_idx[Lc] + (size_t)i * N;
+            // stable compaction of the useful candidates (key > worst elite) into smem
+            uint32_t* s_cnt = (uint32_t*)sm.scratch;     // scratch reused: 33 BestRef >= 9 u32
+            if (threadIdx.x == 0) s_cnt[0] = 0;
+            __syncthreads();
+            for (uint32_t j0 = 0; j0 < C0; j0 += blockDim.x) {
+                const uint32_t j = j0 + threadIdx.x;
+                uint64_t k = 0;
+                uint32_t x = NONE;
+                bool keep = false;
+                if (j < C0) { k = __ldcg(ck + j); x = __ldcg(cx + j); keep = k > thr; }
+                const unsigned m = __ballot_sync(0xFFFFFFFFu, keep);
+                uint32_t pos = 0;
+                if ((threadIdx.x & 31u) == 0 && m) pos = atomicAdd(&s_cnt[0], (uint32_t)__popc(m));
+                pos = __shfl_sync(0xFFFFFFFFu, pos, 0);
+                if (keep) {
+                    const uint32_t r = pos + __popc(m & ((1u << (threadIdx.x & 31u)) - 1u));
+                    sm.skey[r] = k;
+                    sm.sidx[r] = x;
+                }
+            }
+            __syncthreads();
+            const uint32_t C = s_cnt[0];
+            const uint32_t P2 = next_pow2(C < 2 ? 2 : C);
+            for (uint32_t j = C + threadIdx.x; j < P2; j += blockDim.x) { sm.skey[j] = 0ull; sm.sidx[j] = NONE; }
+            bitonic_desc(sm.skey, sm.sidx, P2);
+            trace_mark(a, g, 2);
+            // merged rank of elite r: r + #(candidates with key > ekey[r]);
+            // of candidate j: j + #(elites with key >= ckey[j])  (elites win ties: lower index)
+            for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+                const uint64_t k = sm.ekey[r];
+                uint32_t lo = 0, hi = C;    // first j with skey[j] <= k
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.skey[mid] > k) lo = mid + 1; else hi = mid; }
+                const uint32_t rank = r + lo;
+                if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = r; }
+            }
+            for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
+                const uint64_t k = sm.skey[j];
+                uint32_t lo = 0, hi = E;    // first r with ekey[r] < k
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.ekey[mid] >= k) lo = mid + 1; else hi = mid; }
+                const uint32_t rank = j + lo;
+                if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = sm.sidx[j]; }
+            }
+            __syncthreads();
         }
+        // copy the elites in rank order to slots 0..E-1 of generation g+1 (R18)
+        const uint64_t* rk = general ? sm.skey : sm.okey;
+        const uint32_t* rx = general ? sm.sidx : sm.oidx;
+        uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
+        double* fitn = a.fit[nxt] + (size_t)i * N;
+        for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
+            const uint32_t r = j / W, w = j % W;
+            popn[(size_t)r * W + w] = __ldcg(popc + (size_t)rx[r] * W + w);
+        }
+        for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(rk[r]);
+        if (threadIdx.x == 0) a.tau[cur * I + i] = rk[E - 1];
+    } else if (threadIdx.x == 0) {
+        a.tau[cur * I + i] = ~0ull;    // no elites: no candidate list
     }
-    // a6 mutation, a7 repair, a2 eval of each child (children c0 = A, c0+1 = B)
-    auto finish = [&](Row<WT>& ch_row, uint32_t h) {
-        const uint32_t gid = gid0 + h;
-        const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);
-        if ((uint64_t)rm.x < a.thr_m) row_xor_bit(ch_row, below(rm.y, ch.n - 1));
-        repair(a, ch_row, gid, g);
-        const double f = eval_regs(ch, sP, sO, ch_row, nullptr);
-        const uint32_t slot = c0 + h;
-        row_store(ch_row, popn + (size_t)slot * W, W);
-        fitn[slot] = f;
-        append_if(fkey(f) > tau, ccnt, ckey, cidx, fkey(f), slot);
-        track_best(best, f, slot, ch_row, popn, W);
-    };
-    finish(A, 0);
-    finish(B, 1);
+    if (threadIdx.x == 0) {
+        a.cand_cnt[Lr * I + i] = 0;
+        if (i == 0) { if (general) a.ctl->n_general++; else a.ctl->n_fast++; }
+    }
+    trace_mark(a, g, 3);
 }
 
 // ------------------------------------------------------------------------
-// The cooperative persistent GA kernel
+// The cooperative persistent GA kernel.  CTAs 0..I-1 are island leaders
+// (elite selection, records); the others breed.  One grid barrier per
+// generation: leader(g) runs concurrently with breed(g) because breed(g)
+// needs only generation g and a lagged candidate threshold.
 // ------------------------------------------------------------------------
 template <int WT>
 __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
@@ -838,10 +1126,12 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
     const uint32_t* sP = sm.chain;
     const uint32_t* sO = sm.chain + a.ch.p_words;
     const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I;
-    const uint32_t cpi = gridDim.x / I;                 // CTAs per island
-    const uint32_t my_island = blockIdx.x / cpi;
-    const uint32_t my_local = blockIdx.x % cpi;
-    const bool worker = my_island < I;
+    const uint32_t cpi = (gridDim.x - I) / I;           // worker CTAs per island
+    const bool is_leader = blockIdx.x < I;
+    const uint32_t widx = is_leader ? 0u : blockIdx.x - I;
+    const uint32_t my_island = is_leader ? NONE : widx / cpi;
+    const uint32_t my_local = widx % cpi;
+    const bool worker = !is_leader && my_island < I;
 
     if (a.mode == MODE_INIT) {
         // a1: generation 0 into buffer 0 (all N individuals), partials into parity 0
@@ -849,21 +1139,19 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
             const uint32_t i = my_island;
             uint64_t* pop = a.pop[0] + (size_t)i * N * W;
             double* fit = a.fit[0] + (size_t)i * N;
-            BestRef best{-CUDART_INF, NONE};
+            BestRow<WT> best;
+            best.f = -CUDART_INF;
+            best.idx = NONE;
             for (uint32_t c = my_local * blockDim.x + threadIdx.x; c < N; c += cpi * blockDim.x) {
                 Row<WT> r;
                 init_row(a, r, (a.island_base + i) * N + c);
                 const double f = eval_regs(a.ch, sP, sO, r, nullptr);
                 row_store(r, pop + (size_t)c * W, W);
                 fit[c] = f;
-                track_best(best, f, c, r, pop, W);
+                track_row(best, f, c, r, W);
             }
-            __syncthreads();
-            best = block_best(best, pop, W, sm.scratch);
-            if (threadIdx.x == 0) {
-                a.part_f[(size_t)i * cpi + my_local] = best.f;
-                a.part_idx[(size_t)i * cpi + my_local] = best.idx;
-            }
+            best = block_best_row(best, W, (BestRow<WT>*)sm.scratch);
+            if (threadIdx.x == 0) write_partial(a, (size_t)i * cpi + my_local, best, W);
         }
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             a.ctl->full = 1;
@@ -873,7 +1161,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
             a.ctl->n_fast = 0;
         }
         grid.sync();
-        if (blockIdx.x < I) leader_record(a, blockIdx.x, 0, 0, cpi, a.pop[0], sm);
+        if (is_leader) leader_record<WT>(a, blockIdx.x, 0, 0, cpi, sm);
         return;
     }
 
@@ -881,7 +1169,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
         const uint32_t g = a.g_begin, cur = g & 1u;
         const bool worst = a.mode == MODE_IMPORT;
         general_select(a, a.fit[cur], a.K, worst, sm, grid);
-        if (blockIdx.x < I) {
+        if (is_leader) {
             const uint32_t i = blockIdx.x;
             leader_sort_selected(a, i, a.K, worst, sm);
             uint64_t* pop = a.pop[cur] + (size_t)i * N * W;
@@ -949,107 +1237,59 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
         return;
     }
 
-    // MODE_RUN: generations [g_begin, g_end)
+    // MODE_RUN: generations [g_begin, g_end).  Candidate lists rotate mod 3:
+    // list g%3 holds the candidates of generation g (consumed by leader(g)),
+    // breed(g) appends generation g+1's to list (g+1)%3, leader(g) resets (g+2)%3.
+    const bool first_full = __ldcg(&a.ctl->full) != 0;
     uint32_t g = a.g_begin;
     for (; g < a.g_end; ++g) {
         const uint32_t cur = g & 1u, nxt = cur ^ 1u;
-        const uint64_t* popc_all = a.pop[cur];
-        // ---- phase S: elites of generation g (a3) + record/stall of generation g (a8)
-        bool general = a.ctl->full != 0;
-        if (!general && E > 0)
-            for (uint32_t i = 0; i < I; ++i) general |= __ldcg(&a.cand_cnt[cur * I + i]) > kCandCap;
+        const uint32_t Lc = g % 3u, Lb = (g + 1u) % 3u;
+        bool general = (g == a.g_begin) && first_full;
+        if (!general)
+            for (uint32_t i = 0; i < I; ++i) general |= __ldcg(&a.cand_cnt[Lc * I + i]) > kCandCap;
         general = general && E > 0;
-        if (general) general_select(a, a.fit[cur], E, false, sm, grid);
-        if (blockIdx.x < I) {
-            const uint32_t i = blockIdx.x;
-            leader_record(a, i, g, cur, cpi, popc_all, sm);
-            const uint64_t* popc = popc_all + (size_t)i * N * W;
-            const double* fitc = a.fit[cur] + (size_t)i * N;
-            if (E > 0) {
-                if (general) {
-                    leader_sort_selected(a, i, E, false, sm);
-                } else {
-                    // fast path: previous elites (slots 0..E-1, ranked) merged with the
-                    // children that beat the worst of them (candidates, key > tau)
-                    const uint32_t C = a.cand_cnt[cur * I + i];
-                    const uint32_t P2 = next_pow2(C < 2 ? 2 : C);
-                    const uint64_t* ck = a.cand_key[cur] + (size_t)i * N;
-                    const uint32_t* cx = a.cand_idx[cur] + (size_t)i * N;
-                    for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
-                        sm.skey[j] = j < C ? ck[j] : 0ull;
-                        sm.sidx[j] = j < C ? cx[j] : NONE;
-                    }
-                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) sm.ekey[r] = fkey(fitc[r]);
-                    bitonic_desc(sm.skey, sm.sidx, P2);
-                    // merged rank of elite r: r + #(candidates with key > ekey[r]);
-                    // of candidate j: j + #(elites with key >= ckey[j])  (elites win ties: lower index)
-                    uint64_t* outk = a.sel_key + (size_t)i * kMaxElite;
-                    uint32_t* outx = a.sel_idx + (size_t)i * kMaxElite;
-                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
-                        const uint64_t k = sm.ekey[r];
-                        uint32_t lo = 0, hi = C;    // first j with skey[j] <= k
-                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.skey[mid] > k) lo = mid + 1; else hi = mid; }
-                        const uint32_t rank = r + lo;
-                        if (rank < E) { outk[rank] = k; outx[rank] = r; }
-                    }
-                    for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
-                        const uint64_t k = sm.skey[j];
-                        uint32_t lo = 0, hi = E;    // first r with ekey[r] < k
-                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.ekey[mid] >= k) lo = mid + 1; else hi = mid; }
-                        const uint32_t rank = j + lo;
-                        if (rank < E) { outk[rank] = k; outx[rank] = sm.sidx[j]; }
-                    }
-                    __syncthreads();
-                    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) { sm.skey[r] = outk[r]; sm.sidx[r] = outx[r]; }
-                    __syncthreads();
-                }
-                // copy the elites in rank order to slots 0..E-1 of generation g+1 (R18)
-                uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
-                double* fitn = a.fit[nxt] + (size_t)i * N;
-                for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
-                    const uint32_t r = j / W, w = j % W;
-                    popn[(size_t)r * W + w] = popc[(size_t)sm.sidx[r] * W + w];
-                }
-                for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(sm.skey[r]);
-                if (threadIdx.x == 0) a.tau[i] = sm.skey[E - 1];
-            } else if (threadIdx.x == 0) {
-                a.tau[i] = ~0ull;    // no elites: no candidate list
-            }
-            if (threadIdx.x == 0) {
-                a.cand_cnt[nxt * I + i] = 0;
-                if (i == 0) { if (general) a.ctl->n_general++; else a.ctl->n_fast++; }
-            }
+        uint32_t tau_par = nxt;               // fast path: worst elite of generation g-1 (lagged)
+        if (general) {
+            general_select(a, a.fit[cur], E, false, sm, grid);
+            if (is_leader) leader_phase<WT>(a, blockIdx.x, g, true, cpi, sm);
+            grid.sync();
+            if (__ldcg(&a.ctl->done)) break;
+            tau_par = cur;                    // exact threshold of generation g
+        } else if (is_leader) {
+            leader_phase<WT>(a, blockIdx.x, g, false, cpi, sm);
         }
-        grid.sync();
-        if (__ldcg(&a.ctl->done)) break;
-        if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;
-        // ---- phase B: children of generation g+1 (a4-a7 + a2)
         if (worker) {
+            // a4-a7 + a2: children of generation g+1
             const uint32_t i = my_island;
-            const uint64_t* popc = popc_all + (size_t)i * N * W;
-            const double* fitc = a.fit[cur] + (size_t)i * N;
+            if (threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
+                a.trace[(g - a.g_begin) * 8 + 4] = gtimer();
+            BestRow<WT> best;
+            best.f = -CUDART_INF;
+            best.idx = NONE;
             uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
-            double* fitn = a.fit[nxt] + (size_t)i * N;
-            const uint64_t tau = __ldcg(&a.tau[i]);
-            uint32_t* ccnt = a.cand_cnt + nxt * I + i;
-            uint64_t* ckey = a.cand_key[nxt] + (size_t)i * N;
-            uint32_t* cidx = a.cand_idx[nxt] + (size_t)i * N;
-            const uint32_t pairs = (N - E) / 2;
-            BestRef best{-CUDART_INF, NONE};
-            for (uint32_t q = my_local * blockDim.x + threadIdx.x; q < pairs; q += cpi * blockDim.x)
-                breed_pair<WT>(a, i, q, g, popc, fitc, popn, fitn, sP, sO, tau, ccnt, ckey, cidx, best);
-            __syncthreads();
-            best = block_best(best, popn, W, sm.scratch);
+            breed_children<WT>(a, i, g, my_local, cpi, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * N,
+                               popn, a.fit[nxt] + (size_t)i * N, sP, sO, __ldcg(&a.tau[tau_par * I + i]),
+                               a.cand_cnt + Lb * I + i, a.cand_key[Lb] + (size_t)i * N,
+                               a.cand_idx[Lb] + (size_t)i * N, best);
+            best = block_best_row(best, W, (BestRow<WT>*)sm.scratch);
             if (threadIdx.x == 0) {
-                a.part_f[((size_t)nxt * I + i) * cpi + my_local] = best.f;
-                a.part_idx[((size_t)nxt * I + i) * cpi + my_local] = best.idx;
+                write_partial(a, ((size_t)nxt * I + i) * cpi + my_local, best, W);
+                if (blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
+                    a.trace[(g - a.g_begin) * 8 + 5] = gtimer();
             }
         }
         grid.sync();
+        if (threadIdx.x == 0 && a.trace && g - a.g_begin < a.trace_gens) {
+            if (blockIdx.x == 0) a.trace[(g - a.g_begin) * 8 + 6] = gtimer();
+            if (blockIdx.x == I) a.trace[(g - a.g_begin) * 8 + 7] = gtimer();
+        }
+        if (g == a.g_begin && blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;   // all CTAs read it before this barrier
+        if (__ldcg(&a.ctl->done)) break;
     }
     if (g == a.g_end) {
         // record (and stall) of the last generation of the segment
-        if (blockIdx.x < I) leader_record(a, blockIdx.x, g, g & 1u, cpi, a.pop[g & 1u], sm);
+        if (is_leader) leader_record<WT>(a, blockIdx.x, g, g & 1u, cpi, sm);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->gens_run = g;
 }
@@ -1091,7 +1331,24 @@ __global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
 // ------------------------------------------------------------------------
 static size_t eval_smem(const ChainDev& ch)
 {
-    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
+    const size_t tile = ch.W <= 16 ? (size_t)(2 * ch.W + 1) * 4 : (size_t)(ch.W | 1u) * 8;
+    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * tile;
+}
+
+template <int W>
+static void* eval_fn_w() { return (void*)eval_batch_w_kernel<W>; }
+
+static void* eval_pick(uint32_t W)
+{
+    switch (W) {
+    case 1: return eval_fn_w<1>();   case 2: return eval_fn_w<2>();   case 3: return eval_fn_w<3>();
+    case 4: return eval_fn_w<4>();   case 5: return eval_fn_w<5>();   case 6: return eval_fn_w<6>();
+    case 7: return eval_fn_w<7>();   case 8: return eval_fn_w<8>();   case 9: return eval_fn_w<9>();
+    case 10: return eval_fn_w<10>(); case 11: return eval_fn_w<11>(); case 12: return eval_fn_w<12>();
+    case 13: return eval_fn_w<13>(); case 14: return eval_fn_w<14>(); case 15: return eval_fn_w<15>();
+    case 16: return eval_fn_w<16>();
+    default: return (void*)eval_batch_kernel;
+    }
 }
 
 cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out, cudaStream_t st,
@@ -1099,19 +1356,24 @@ cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t
 {
     if (n_cand == 0) return cudaSuccess;
     const size_t sm = eval_smem(ch);
-    cudaError_t e = cudaFuncSetAttribute(eval_batch_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    void* fn = eval_pick(ch.W);
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, eval_batch_kernel, kEvalWarps * 32, sm);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kEvalWarps * 32, sm);
     if (e != cudaSuccess) return e;
     if (per_sm < 1) per_sm = 1;
     const uint64_t tiles = (n_cand + 31) / 32;
     uint64_t grid = (uint64_t)per_sm * num_sms;
     const uint64_t need = (tiles + kEvalWarps - 1) / kEvalWarps;
     if (grid > need) grid = need;
-    eval_batch_kernel<<<(unsigned)grid, kEvalWarps * 32, sm, st>>>(ch, bits, n_cand, out);
+    ChainDev c = ch;
+    const uint64_t* b = bits;
+    double* o = out;
+    void* args[] = {&c, &b, &n_cand, &o};
+    e = cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kEvalWarps * 32), args, sm, st);
     if (launches) ++*launches;
-    return cudaGetLastError();
+    return e;
 }
 
 size_t ga_smem_bytes(const GaArgs& a) { return smem_layout(a, nullptr, nullptr); }

@@ -1,0 +1,36 @@
+"""Minimal drivers for ncu captures (one GPU): `eval` runs split_eval_batch on C5,
+`ga` runs split_ga_run on C2.  Not a benchmark (numbers under ncu are not bench values)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_icpp_luoyww0023_b200 import split as S  # noqa: E402
+from paper_conf_icpp_luoyww0023_b200 import workloads as wl  # noqa: E402
+
+
+def main(what: str, reps: int = 3, gens: int = 500):
+    torch.cuda.set_device(0)
+    st = torch.cuda.current_stream()
+    if what == "eval":
+        lat, ovh = wl.chain("synthetic_1024")
+        n_cand = 1 << 24
+        h = S.SplitGA(lat, ovh, pop_size=4, n_elite=0, k_min=2, k_max=32, stream=st)
+        bits = torch.from_numpy(wl.uniform_k_population_fast(len(lat), n_cand, seed=20230807).view(np.int64)).cuda()
+        out = torch.empty(n_cand, dtype=torch.float64, device="cuda")
+        for _ in range(reps):
+            h.eval_batch(bits, n_cand, out)
+        torch.cuda.synchronize()
+    else:
+        lat, ovh = wl.chain("resnet50_175")
+        h = S.SplitGA(lat, ovh, pop_size=65536, n_elite=1024, k_min=2, k_max=32, stream=st)
+        for i in range(reps):
+            r = h.run(gens, i)
+        print(r["fitness"], h.last_run_stats())
+    h.close()
+
+
+if __name__ == "__main__":
+    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 3, int(sys.argv[3]) if len(sys.argv) > 3 else 500)
