@@ -361,6 +361,20 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     uint32_t sc = std::max<uint32_t>(pow2_at_least(kCandCap), pow2_at_least(std::max<uint32_t>(a.E, 2)));
     if (migrate) sc = std::max(sc, pow2_at_least((p.n_islands - 1) * a.K));
     a.sort_cap = sc;
+    a.Ns = (a.N + 3u) & ~3u;
+    // size the per-CTA partial arrays for the largest grid the launch bounds allow,
+    // then take the real co-resident grid from the occupancy calculator
+    {
+        const uint32_t grid_max = (uint32_t)(ga_max_blocks_per_sm(h->W) * h->num_sms);
+        if (grid_max < 2 * a.I) {
+            free_all(h);
+            delete h;
+            return fail(SPLIT_E_INVAL, "too many islands per device for %d SMs", h->num_sms);
+        }
+        a.cpi = (grid_max - a.I) / a.I;
+        a.cpi_pad = (a.cpi + 3u) & ~3u;
+        a.stage_bits = (size_t)a.cpi_pad * h->W * 8 <= 16384 ? 1u : 0u;
+    }
     if (ga_smem_bytes(a) > 227 * 1024) {
         free_all(h);
         delete h;
@@ -369,35 +383,35 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     }
     cudaError_t ge;
     h->grid = ga_grid(a, h->num_sms, &ge);
-    if (ge != cudaSuccess || h->grid < (int)a.I) {
+    if (ge != cudaSuccess || h->grid < 2 * (int)a.I) {
         free_all(h);
         delete h;
-        return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s", cudaGetErrorString(ge));
+        return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s (grid %d)", cudaGetErrorString(ge), h->grid);
     }
-    if (h->grid < 2 * (int)a.I) {
-        free_all(h);
-        delete h;
-        return fail(SPLIT_E_INVAL, "grid %d too small for %u islands", h->grid, a.I);
-    }
-    h->cpi = (uint32_t)(h->grid - (int)a.I) / a.I;
-    const size_t IN = (size_t)a.I * a.N;
+    a.cpi = (uint32_t)(h->grid - (int)a.I) / a.I;     // <= the sizing value; cpi_pad keeps its value
+    h->cpi = a.cpi;
+    const size_t IN = (size_t)a.I * a.N, INs = (size_t)a.I * a.Ns;
     for (int b = 0; b < 2; ++b) {
         TRY(dalloc(h, &a.pop[b], IN * h->W));
-        TRY(dalloc(h, &a.fit[b], IN));
+        TRY(dalloc(h, &a.fit[b], INs));
     }
     for (int b = 0; b < 3; ++b) {
-        TRY(dalloc(h, &a.cand_key[b], IN));
-        TRY(dalloc(h, &a.cand_idx[b], IN));
+        TRY(dalloc(h, &a.cand_key[b], INs));
+        TRY(dalloc(h, &a.cand_idx[b], INs));
     }
-    TRY(dalloc(h, &a.cand_cnt, 3 * (size_t)a.I));
+    TRY(dalloc(h, &a.cand_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4));   // 16-byte chunks readable
+    TRY(dalloc(h, &a.rc_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4));
+    for (int b = 0; b < 3; ++b) TRY(dalloc(h, &a.rc_idx[b], INs));
+    TRY(dalloc(h, &a.snap_f, 2 * (size_t)a.I));
+    TRY(dalloc(h, &a.snap_bits, 2 * (size_t)a.I * h->W));
     TRY(dalloc(h, &a.sel_key, (size_t)a.I * kMaxElite));
     TRY(dalloc(h, &a.sel_idx, (size_t)a.I * kMaxElite));
     TRY(dalloc(h, &a.sel_cnt, a.I));
     TRY(dalloc(h, &a.tau, 2 * (size_t)a.I));
     TRY(dalloc(h, &a.ghist, 3 * (size_t)a.I * 256));
-    TRY(dalloc(h, &a.part_f, 2 * (size_t)a.I * h->cpi));
-    TRY(dalloc(h, &a.part_idx, 2 * (size_t)a.I * h->cpi));
-    TRY(dalloc(h, &a.part_bits, 2 * (size_t)a.I * h->cpi * h->W));
+    TRY(dalloc(h, &a.part_f, 2 * (size_t)a.I * a.cpi_pad));
+    TRY(dalloc(h, &a.part_idx, 2 * (size_t)a.I * a.cpi_pad));
+    TRY(dalloc(h, &a.part_bits, 2 * (size_t)a.I * a.cpi_pad * h->W));
     TRY(dalloc(h, &a.rec_f, a.I));
     TRY(dalloc(h, &a.rec_bits, (size_t)a.I * h->W));
     TRY(dalloc(h, &a.rec_gen, a.I));
@@ -411,7 +425,7 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     TRY(dalloc(h, &h->d_recpack, (size_t)a.I_total * (h->W + 2)));
     if (getenv("SPLIT_TRACE")) {
         h->trace_gens = 64;
-        TRY(dalloc(h, &h->d_trace, (size_t)h->trace_gens * 8));
+        TRY(dalloc(h, &h->d_trace, (size_t)h->trace_gens * 16));
     }
     for (int i = 0; i < 4; ++i) {
         cudaError_t e = cudaEventCreate(&h->ev[i]);
@@ -492,7 +506,7 @@ static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
     a.trace_gens = h->trace_gens;
     a.g_begin = g0;
     a.g_end = g1;
-    cudaError_t e = launch_ga(a, h->stream, h->num_sms, &h->stats.launches);
+    cudaError_t e = launch_ga(a, h->grid, h->stream, &h->stats.launches);
     if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "GA kernel (mode %u): %s", mode, cudaGetErrorString(e));
     return SPLIT_OK;
 }
@@ -573,6 +587,7 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     h->stats = split_run_stats{};
     CU(cudaMemsetAsync(a.rec_valid, 0, a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.cand_cnt, 0, 3 * a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.rc_cnt, 0, 3 * a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.sel_cnt, 0, a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.ghist, 0, 3 * a.I * 256 * 4, h->stream));
     CU(cudaMemsetAsync(a.tau, 0xFF, 2 * a.I * 8, h->stream));
@@ -660,13 +675,15 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     h->last_gen = gens_run;
     h->have_pop = true;
     if (h->d_trace) {
-        std::vector<unsigned long long> tr((size_t)h->trace_gens * 8);
+        std::vector<unsigned long long> tr((size_t)h->trace_gens * 16);
         CU(cudaMemcpy(tr.data(), h->d_trace, tr.size() * 8, cudaMemcpyDeviceToHost));
         if (FILE* f = fopen(getenv("SPLIT_TRACE"), "w")) {
-            fprintf(f, "gen,lead_start,lead_record,lead_sort,lead_end,work_start,work_end,lead_sync,work_sync\n");
+            fprintf(f, "gen,lead_start,lead_record,lead_sort,lead_end,work_start,work_end,lead_sync,work_sync,"
+                       "b_tourn,b_rows,b_repair,b_eval,b_store,w_loopend,w_allwarps,lead_loaded\n");
+            CU(cudaMemset(h->d_trace, 0, tr.size() * 8));
             for (uint32_t g = 0; g < h->trace_gens; ++g) {
                 fprintf(f, "%u", g);
-                for (int j = 0; j < 8; ++j) fprintf(f, ",%llu", tr[(size_t)g * 8 + j]);
+                for (int j = 0; j < 16; ++j) fprintf(f, ",%llu", tr[(size_t)g * 16 + j]);
                 fprintf(f, "\n");
             }
             fclose(f);
@@ -686,7 +703,8 @@ extern "C" int split_ga_population(split_ga_t* h, uint32_t island, uint64_t* bit
     const size_t N = h->ga.N, W = h->W;
     if (bits_host)
         CU(cudaMemcpyAsync(bits_host, h->ga.pop[b] + island * N * W, N * W * 8, cudaMemcpyDeviceToHost, h->stream));
-    if (fit_host) CU(cudaMemcpyAsync(fit_host, h->ga.fit[b] + island * N, N * 8, cudaMemcpyDeviceToHost, h->stream));
+    if (fit_host)
+        CU(cudaMemcpyAsync(fit_host, h->ga.fit[b] + island * (size_t)h->ga.Ns, N * 8, cudaMemcpyDeviceToHost, h->stream));
     CU(cudaStreamSynchronize(h->stream));
     return SPLIT_OK;
 }

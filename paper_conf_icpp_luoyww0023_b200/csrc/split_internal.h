@@ -9,6 +9,7 @@ namespace splitga {
 constexpr uint32_t kMaxLocalIslands = 16;   // islands batched on one device
 constexpr uint32_t kMaxElite = 1024;        // E and K (v1 bound)
 constexpr uint32_t kCandCap = 2048;         // fast elite merge handles up to this many candidates
+constexpr uint32_t kRecWin = 256;           // record-candidate entries staged by TMA
 constexpr uint32_t kMaxWords = 64;          // n_ops <= 4097
 constexpr uint32_t kBlock = 256;            // threads per CTA of the GA kernel
 
@@ -23,7 +24,7 @@ struct Ctl {
     uint32_t last_improve;  // generation of the last strict improvement (single island)
     double f_improve;       // record fitness at the last improvement
     uint32_t n_general, n_fast;
-    uint32_t pad[2];
+    uint32_t redo[2];       // redo[g&1] == g+1: a leader's candidate list overflowed in generation g
 };
 
 // Chain staged for the kernels: P[0..n] (u32, exclusive prefix of the latencies)
@@ -48,9 +49,12 @@ struct GaArgs {
     uint32_t mode, g_begin, g_end;     // MODE_*, generation range of a RUN segment
     uint32_t stall_in_kernel;          // single global island: stall checked every generation
     uint32_t sort_cap;                 // power of two, entries the leader can sort in smem
+    uint32_t Ns;                       // island stride of fit/cand arrays (N rounded up to 4)
+    uint32_t cpi, cpi_pad;             // worker CTAs per island; partial-array stride (mult. of 4)
+    uint32_t stage_bits;               // leader stages partial bits in smem (small W)
     uint64_t* pop[2];                  // [I][N][W]
-    double* fit[2];                    // [I][N]
-    uint64_t* cand_key[3];             // [I][N]   candidates of generation g (list g%3)
+    double* fit[2];                    // [I][Ns]
+    uint64_t* cand_key[3];             // [I][Ns]  candidates of generation g (list g%3)
     uint32_t* cand_idx[3];
     uint32_t* cand_cnt;                // [3][I]
     uint64_t* sel_key;                 // [I][kMaxElite] general-select / elite output
@@ -58,15 +62,19 @@ struct GaArgs {
     uint32_t* sel_cnt;                 // [I]
     uint64_t* tau;                     // [2][I] key of the worst elite of generation g (parity g&1)
     uint32_t* ghist;                   // [3][I][256]
-    double* part_f;                    // [2][I][cpi] per-CTA best child
+    double* part_f;                    // [2][I][cpi_pad] per-CTA best child
     uint32_t* part_idx;
-    uint64_t* part_bits;               // [2][I][cpi][W] bits of each per-CTA best
+    uint64_t* part_bits;               // [2][I][cpi_pad][W] bits of each per-CTA best
     double* rec_f;                     // [I] island records
     uint64_t* rec_bits;                // [I][W]
     uint32_t* rec_gen;                 // [I]
     uint32_t* rec_valid;               // [I]
     uint64_t* mig_bits;                // [I_total][K][W]
     double* mig_f;                     // [I_total][K]
+    uint32_t* rc_cnt;                  // [3][I] record-candidate lists (children that beat a
+    uint32_t* rc_idx[3];               //        snapshot of the island record), rotation as cand_*
+    double* snap_f;                    // [2][I] record snapshots (parity g&1), read by breed(g+1)
+    uint64_t* snap_bits;               // [2][I][W]
     Ctl* ctl;
     unsigned long long* trace;         // optional phase timestamps (SPLIT_TRACE), [trace_gens][8]
     uint32_t trace_gens;
@@ -76,9 +84,10 @@ struct GaArgs {
 cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out,
                               cudaStream_t st, int num_sms, uint64_t* launches);
 // Cooperative persistent GA kernel; grid = blocks_per_sm * num_sms.
-cudaError_t launch_ga(const GaArgs& a, cudaStream_t st, int num_sms, uint64_t* launches);
+cudaError_t launch_ga(const GaArgs& a, int grid, cudaStream_t st, uint64_t* launches);
 size_t ga_smem_bytes(const GaArgs& a);
 int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err);
+int ga_max_blocks_per_sm(uint32_t W);
 cudaError_t launch_eval_stats(const ChainDev& ch, const uint64_t* bits, int64_t* stats_out /*[5]*/,
                               double* f_out, cudaStream_t st);
 cudaError_t launch_selftest_philox(const uint32_t* in, uint32_t n, uint32_t* out, cudaStream_t st);

@@ -118,8 +118,23 @@ __device__ __forceinline__ void trace_mark(const GaArgs& a, uint32_t g, uint32_t
 {
     if (!a.trace || threadIdx.x != 0 || blockIdx.x != 0) return;
     const uint32_t gi = g - a.g_begin;
-    if (gi < a.trace_gens) a.trace[gi * 8 + slot] = gtimer();
+    if (gi < a.trace_gens) a.trace[gi * 16 + slot] = gtimer();
 }
+
+// asynchronous global->shared copies (LDGSTS), no register staging
+__device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"((uint32_t)__cvta_generic_to_shared(smem_dst)),
+                 "l"(gsrc)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(smem_dst)),
+                 "l"(gsrc)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 // order-preserving u64 key of a fitness (larger f -> larger key)
 __device__ __forceinline__ uint64_t fkey(double f)
@@ -642,7 +657,7 @@ __device__ __forceinline__ void append_if(bool pred, uint32_t* cnt, uint64_t* ke
     base = __shfl_sync(act, base, leader);
     if (pred) {
         const uint32_t r = __popc(m & ((1u << lane) - 1u));
-        keys[base + r] = key;
+        if (keys) keys[base + r] = key;
         idxs[base + r] = idx;
     }
 }
@@ -658,17 +673,29 @@ struct SelState {
     uint32_t done;
 };
 
+struct RecCache {
+    double f, f_improve;
+    uint32_t valid, gen, last_improve, done;
+    uint64_t bits[1];     // W words (allocated to W)
+};
+
 struct Smem {
     uint32_t* chain;
-    uint64_t* mbar;
+    uint64_t* mbar;       // [0]: chain staging, [1]: leader loads (reused every generation)
     uint32_t* hist;       // [I][256]
     SelState* sel;        // [I]
-    BestRef* scratch;     // [33]
+    BestRef* scratch;     // 33 BestRow<WT>
+    uint32_t* misc;       // 32 words
+    uint32_t* rcw;        // [kRecWin] window of the record-candidate list
     uint64_t* skey;       // [sort_cap]
     uint32_t* sidx;       // [sort_cap]
     uint64_t* ekey;       // [kMaxElite]
     uint64_t* okey;       // [kMaxElite] merged elites (fast path)
     uint32_t* oidx;
+    RecCache* rec;        // leader: island record + stall state, cached for the whole launch
+    double* pf;           // [cpi_pad] staged partial bests (leader)
+    uint32_t* pi;
+    uint64_t* pb;         // [cpi_pad][W] when a.stage_bits
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
@@ -685,14 +712,61 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take(16); if (s) s->mbar = (uint64_t*)p;
     p = take((size_t)a.I * 256 * 4); if (s) s->hist = (uint32_t*)p;
     p = take((size_t)a.I * sizeof(SelState)); if (s) s->sel = (SelState*)p;
-    p = take(33 * (16 + 8 * (size_t)wt_of(a.ch.W))); if (s) s->scratch = (BestRef*)p;   // 33 BestRow<WT>
+    p = take(33 * (16 + 8 * (size_t)wt_of(a.ch.W))); if (s) s->scratch = (BestRef*)p;
+    p = take(128); if (s) s->misc = (uint32_t*)p;
+    p = take((size_t)kRecWin * 4); if (s) s->rcw = (uint32_t*)p;
     p = take((size_t)a.sort_cap * 8); if (s) s->skey = (uint64_t*)p;
     p = take((size_t)a.sort_cap * 4); if (s) s->sidx = (uint32_t*)p;
-    p = take((size_t)kMaxElite * 8); if (s) s->ekey = (uint64_t*)p;
+    p = take((size_t)kMaxElite * 8 + 16); if (s) s->ekey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 8); if (s) s->okey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 4); if (s) s->oidx = (uint32_t*)p;
+    p = take(sizeof(RecCache) + 8 * (size_t)a.ch.W); if (s) s->rec = (RecCache*)p;
+    p = take((size_t)a.cpi_pad * 8); if (s) s->pf = (double*)p;
+    p = take((size_t)a.cpi_pad * 4); if (s) s->pi = (uint32_t*)p;
+    p = take(a.stage_bits ? (size_t)a.cpi_pad * a.ch.W * 8 : 16); if (s) s->pb = (uint64_t*)p;
     return off;
 }
+
+// ------------------------------------------------------------------------
+// mbarrier + TMA bulk copies (cp.async.bulk) for the leader's loads
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* mbar, uint32_t bytes)
+{
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* mbar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t parity)
+{
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(ok)
+            : "r"(smem_u32(mbar)), "r"(parity)
+            : "memory");
+    }
+}
+// bytes: multiple of 16; src/dst 16-byte aligned
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* mbar)
+{
+    const uint32_t d = smem_u32(dst), b = smem_u32(mbar);
+    for (uint32_t off = 0; off < bytes; off += 32768u) {
+        const uint32_t n = (bytes - off < 32768u) ? (bytes - off) : 32768u;
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d + off),
+                     "l"((const char*)src + off), "r"(n), "r"(b)
+                     : "memory");
+    }
+}
+__host__ __device__ inline uint32_t round16(uint32_t bytes) { return (bytes + 15u) & ~15u; }
 
 // composite of element i of an island: desc order (elite/export) -> (key, ~idx);
 // worst order (import) -> (~key, idx).  Larger composite = selected first.
@@ -726,7 +800,7 @@ __device__ __forceinline__ bool sel_selected(uint64_t hi, uint32_t lo, const Sel
 
 // General top-Ksel per local island by 96-bit radix select (MSB first, 8-bit
 // digits), all CTAs cooperating with grid barriers.  Output (unsorted):
-// sel_key/sel_idx[i][0..Ksel) with sel_cnt[i] == Ksel.  fit: [I][N].
+// sel_key/sel_idx[i][0..Ksel) with sel_cnt[i] == Ksel.  fit: [I][Ns].
 __device__ void general_select(const GaArgs& a, const double* fit, uint32_t Ksel, bool worst, const Smem& sm,
                                cg::grid_group& grid)
 {
@@ -754,7 +828,7 @@ __device__ void general_select(const GaArgs& a, const double* fit, uint32_t Ksel
             const SelState& s = sm.sel[i];
             if (s.done) continue;
             uint64_t hi; uint32_t lo;
-            composite(fit[e], idx, worst, hi, lo);
+            composite(__ldcg(fit + (size_t)i * a.Ns + idx), idx, worst, hi, lo);
             if (sel_match(hi, lo, s)) atomicAdd(&sm.hist[i * 256 + sel_digit(hi, lo, s.d)], 1u);
         }
         __syncthreads();
@@ -815,7 +889,7 @@ __device__ void general_select(const GaArgs& a, const double* fit, uint32_t Ksel
     for (uint64_t e = gtid; e < total; e += gstride) {
         const uint32_t i = (uint32_t)(e / N), idx = (uint32_t)(e % N);
         const SelState s = sm.sel[i];
-        const double f = fit[e];
+        const double f = __ldcg(fit + (size_t)i * a.Ns + idx);
         uint64_t hi; uint32_t lo;
         composite(f, idx, worst, hi, lo);
         const bool take = (Ksel > 0) && sel_selected(hi, lo, s);
@@ -854,18 +928,34 @@ __device__ void leader_sort_selected(const GaArgs& a, uint32_t i, uint32_t Ksel,
     if (threadIdx.x == 0) a.sel_cnt[i] = 0;
 }
 
-// Leader CTA: record update of island i from the per-CTA partial bests of
-// generation g (f, index and bits, in part_*), and the single-island stall
-// rule (R11).
+
+// Leader CTA: load island i's record and stall state into shared memory once
+// per launch; every update writes through to global memory for the host.
+__device__ void rec_load(const GaArgs& a, uint32_t i, const Smem& sm)
+{
+    if (threadIdx.x == 0) {
+        RecCache* r = sm.rec;
+        r->valid = __ldcg(a.rec_valid + i);
+        r->f = __ldcg(a.rec_f + i);
+        r->gen = __ldcg(a.rec_gen + i);
+        for (uint32_t w = 0; w < a.ch.W; ++w) r->bits[w] = __ldcg(a.rec_bits + (size_t)i * a.ch.W + w);
+        r->f_improve = __ldcg(&a.ctl->f_improve);
+        r->last_improve = __ldcg(&a.ctl->last_improve);
+        r->done = 0;
+    }
+    __syncthreads();
+}
+
+// thread-level best over this thread's share of the per-CTA partials, from global
 template <int WT>
-__device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t parity, uint32_t cpi, const Smem& sm)
+__device__ __forceinline__ BestRow<WT> load_partials(const GaArgs& a, uint32_t i, uint32_t parity)
 {
     const uint32_t W = a.ch.W;
     BestRow<WT> v;
     v.f = -CUDART_INF;
     v.idx = NONE;
-    const size_t base = ((size_t)parity * a.I + i) * cpi;
-    for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x) {
+    const size_t base = ((size_t)parity * a.I + i) * a.cpi_pad;
+    for (uint32_t j = threadIdx.x; j < a.cpi; j += blockDim.x) {
         BestRow<WT> o;
         o.f = __ldcg(a.part_f + base + j);
         o.idx = __ldcg(a.part_idx + base + j);
@@ -873,45 +963,227 @@ __device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t 
         for (int w = 0; w < WT; ++w) o.r.w[w] = (w < (int)W) ? __ldcg(a.part_bits + (base + j) * W + w) : 0ull;
         if (better_row(o, v, W)) v = o;
     }
-    v = block_best_row(v, W, (BestRow<WT>*)sm.scratch);
+    return v;
+}
+
+// Record update of island i with the best candidate of generation g (block-
+// reduced when `reduce`), the single-island stall rule (R11), and the snapshot
+// of the record that breed(g+1) filters against.
+template <int WT>
+__device__ void record_apply(const GaArgs& a, uint32_t i, uint32_t g, BestRow<WT> v, bool reduce, const Smem& sm)
+{
+    const uint32_t W = a.ch.W;
+    if (reduce) v = block_best_row(v, W, (BestRow<WT>*)sm.scratch);
     if (threadIdx.x == 0) {
+        RecCache* rc = sm.rec;
         bool upd = false;
-        if (v.idx != NONE) {
-            if (!a.rec_valid[i]) upd = true;
-            else if (v.f != a.rec_f[i]) upd = v.f > a.rec_f[i];
+        if (reduce && v.idx != NONE) {
+            if (!rc->valid) upd = true;
+            else if (v.f != rc->f) upd = v.f > rc->f;
             else {
                 BestRow<WT> rec;
                 rec.f = v.f;
                 rec.idx = 0;
 #pragma unroll
-                for (int w = 0; w < WT; ++w) rec.r.w[w] = (w < (int)W) ? a.rec_bits[(size_t)i * W + w] : 0ull;
+                for (int w = 0; w < WT; ++w) rec.r.w[w] = (w < (int)W) ? rc->bits[w] : 0ull;
                 upd = better_row(v, rec, W);
             }
         }
         if (upd) {
+            rc->f = v.f;
+            rc->gen = g;
+            rc->valid = 1;
             a.rec_f[i] = v.f;
             a.rec_gen[i] = g;
             a.rec_valid[i] = 1;
 #pragma unroll
             for (int w = 0; w < WT; ++w)
-                if (w < (int)W) a.rec_bits[(size_t)i * W + w] = v.r.w[w];
+                if (w < (int)W) { rc->bits[w] = v.r.w[w]; a.rec_bits[(size_t)i * W + w] = v.r.w[w]; }
         }
+        // snapshot of generation g's record for breed(g+1) (parity g&1)
+        const uint32_t sp = (g & 1u) * a.I + i;
+        a.snap_f[sp] = rc->valid ? rc->f : -CUDART_INF;
+        for (uint32_t w = 0; w < W; ++w) a.snap_bits[(size_t)sp * W + w] = rc->valid ? rc->bits[w] : ~0ull;
         if (a.stall_in_kernel && i == 0) {
-            Ctl* c = a.ctl;
             if (g == 0) {
-                c->f_improve = a.rec_f[0];
-                c->last_improve = 0;
+                rc->f_improve = rc->f;
+                rc->last_improve = 0;
             } else {
-                if (a.rec_f[0] > c->f_improve) { c->f_improve = a.rec_f[0]; c->last_improve = g; }
-                if (a.stall > 0 && g - c->last_improve >= a.stall) c->done = 1;
+                if (rc->f > rc->f_improve) { rc->f_improve = rc->f; rc->last_improve = g; }
+                if (a.stall > 0 && g - rc->last_improve >= a.stall) { rc->done = 1; a.ctl->done = 1; }
             }
+            a.ctl->f_improve = rc->f_improve;
+            a.ctl->last_improve = rc->last_improve;
         }
     }
     __syncthreads();
 }
 
+// INIT: record of generation 0 from the per-CTA partial bests; both snapshots
+template <int WT>
+__device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t parity, const Smem& sm)
+{
+    record_apply<WT>(a, i, g, load_partials<WT>(a, i, parity), true, sm);
+    if (threadIdx.x == 0) {
+        const uint32_t sp = (1u - (g & 1u)) * a.I + i;
+        a.snap_f[sp] = a.snap_f[(g & 1u) * a.I + i];
+        for (uint32_t w = 0; w < a.ch.W; ++w)
+            a.snap_bits[(size_t)sp * a.ch.W + w] = a.snap_bits[((size_t)(g & 1u) * a.I + i) * a.ch.W + w];
+    }
+}
+
+// Record of generation g from the record-candidate list (children that beat a
+// snapshot of an earlier record, list g%3).  R entries, the first kRecWin of
+// them staged in sm.rcw; rows and fitness are read from generation g.
+template <int WT>
+__device__ void leader_record_list(const GaArgs& a, uint32_t i, uint32_t g, uint32_t R, bool staged,
+                                   const Smem& sm)
+{
+    const uint32_t W = a.ch.W, L = g % 3u, cur = g & 1u;
+    const uint64_t* popc = a.pop[cur] + (size_t)i * a.N * W;
+    const double* fitc = a.fit[cur] + (size_t)i * a.Ns;
+    const uint32_t* lst = a.rc_idx[L] + (size_t)i * a.Ns;
+    BestRow<WT> v;
+    v.f = -CUDART_INF;
+    v.idx = NONE;
+    for (uint32_t r = threadIdx.x; r < R; r += blockDim.x) {
+        const uint32_t slot = (staged && r < kRecWin) ? sm.rcw[r] : __ldcg(lst + r);
+        BestRow<WT> o;
+        o.f = __ldcg(fitc + slot);
+        o.idx = slot;
+#pragma unroll
+        for (int w = 0; w < WT; ++w) o.r.w[w] = (w < (int)W) ? __ldcg(popc + (size_t)slot * W + w) : 0ull;
+        if (better_row(o, v, W)) v = o;
+    }
+    record_apply<WT>(a, i, g, v, R > 0, sm);
+}
+
+// Copy the ranked elites (keys rk, indices rx into generation g) to slots
+// 0..E-1 of generation g+1 (R18) and publish the worst elite's key.
+__device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, const uint64_t* rk, const uint32_t* rx)
+{
+    const uint32_t W = a.ch.W, N = a.N, E = a.E;
+    const uint32_t cur = g & 1u, nxt = cur ^ 1u;
+    const uint64_t* popc = a.pop[cur] + (size_t)i * N * W;
+    uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
+    double* fitn = a.fit[nxt] + (size_t)i * a.Ns;
+    for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
+        const uint32_t r = j / W, w = j % W;
+        popn[(size_t)r * W + w] = __ldcg(popc + (size_t)rx[r] * W + w);
+    }
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(rk[r]);
+    if (threadIdx.x == 0) a.tau[cur * a.I + i] = rk[E - 1];
+}
+
+// Leader, general path: the radix select already gathered the E best of
+// generation g; sort them and place them.
+__device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm)
+{
+    leader_sort_selected(a, i, a.E, false, sm);
+    leader_copy_elites(a, i, g, sm.skey, sm.sidx);
+    __syncthreads();
+}
+
+// Leader, fast path of generation g.  One mbarrier gathers (TMA bulk copies)
+// the per-CTA partial bests, the previous elites' fitness (slots 0..E-1 of
+// generation g, ranked) and the candidate children (a superset of those that
+// beat the worst previous elite).  Then: record + stall (a8), merge of the
+// elites with the sorted candidates (a3), elite copy.  If the candidate list
+// overflowed, the leader only stamps ctl->redo[g&1] and every CTA runs the
+// general path after the barrier.
+template <int WT>
+__device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm, uint32_t& mph)
+{
+    const uint32_t W = a.ch.W, Ns = a.Ns, E = a.E, I = a.I, cpi = a.cpi, cpp = a.cpi_pad;
+    const uint32_t cur = g & 1u, Lc = g % 3u, Lr = (g + 2u) % 3u;
+    trace_mark(a, g, 0);
+    if (threadIdx.x == 0) {
+        // one TMA batch: record-candidate count (its 16-byte chunk) + a window of the
+        // list, previous elites' fitness, candidate count chunk + a window of the list
+        const uint32_t cnt_off = Lc * I + i;
+        const uint32_t win = Ns < kCandCap ? Ns : kCandCap;      // Ns is a multiple of 4
+        const uint32_t rwin = Ns < kRecWin ? Ns : kRecWin;
+        const uint32_t b = 16u + rwin * 4u + (E > 0 ? round16(E * 8u) + 16u + win * 12u : 0u);
+        mbar_arrive_expect_tx(sm.mbar + 1, b);
+        bulk_g2s(sm.misc + 16, a.rc_cnt + (cnt_off & ~3u), 16u, sm.mbar + 1);
+        bulk_g2s(sm.rcw, a.rc_idx[Lc] + (size_t)i * Ns, rwin * 4u, sm.mbar + 1);
+        if (E > 0) {
+            bulk_g2s(sm.ekey, a.fit[cur] + (size_t)i * Ns, round16(E * 8u), sm.mbar + 1);
+            bulk_g2s(sm.misc + 4, a.cand_cnt + (cnt_off & ~3u), 16u, sm.mbar + 1);
+            bulk_g2s(sm.skey, a.cand_key[Lc] + (size_t)i * Ns, win * 8u, sm.mbar + 1);
+            bulk_g2s(sm.sidx, a.cand_idx[Lc] + (size_t)i * Ns, win * 4u, sm.mbar + 1);
+        }
+    }
+    mbar_wait(sm.mbar + 1, mph);
+    mph ^= 1u;
+    if (a.trace && threadIdx.x == 0 && blockIdx.x == 0 && g - a.g_begin < a.trace_gens)
+        a.trace[(g - a.g_begin) * 16 + 15] = gtimer();
+    const uint32_t C0 = E > 0 ? sm.misc[4 + ((Lc * I + i) & 3u)] : 0u;
+    const uint32_t R = sm.misc[16 + ((Lc * I + i) & 3u)];
+    const bool ok = C0 <= kCandCap;
+    // a8: record of generation g
+    leader_record_list<WT>(a, i, g, R, true, sm);
+    trace_mark(a, g, 1);
+    if (threadIdx.x == 0) { a.cand_cnt[Lr * I + i] = 0; a.rc_cnt[Lr * I + i] = 0; }
+    if (E == 0) {
+        if (threadIdx.x == 0) a.tau[cur * I + i] = ~0ull;
+        return;
+    }
+    if (!ok) {
+        if (threadIdx.x == 0) a.ctl->redo[cur] = g + 1;            // generation-stamped: no reset needed
+        return;
+    }
+    // a3 fast path: previous elites (ranked) + candidates that beat the worst of them
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) sm.ekey[r] = fkey(__longlong_as_double((long long)sm.ekey[r]));
+    if (threadIdx.x == 0) sm.misc[2] = 0;
+    __syncthreads();
+    const uint64_t thr = sm.ekey[E - 1];
+    for (uint32_t j0 = 0; j0 < C0; j0 += blockDim.x) {          // in-place compaction
+        const uint32_t j = j0 + threadIdx.x;
+        const uint64_t k = j < C0 ? sm.skey[j] : 0ull;
+        const uint32_t x = j < C0 ? sm.sidx[j] : NONE;
+        const bool keep = (j < C0) && k > thr;
+        const unsigned m = __ballot_sync(0xFFFFFFFFu, keep);
+        __syncthreads();                                            // the chunk is read before any write
+        uint32_t pos = 0;
+        if ((threadIdx.x & 31u) == 0 && m) pos = atomicAdd(&sm.misc[2], (uint32_t)__popc(m));
+        pos = __shfl_sync(0xFFFFFFFFu, pos, 0);
+        if (keep) {
+            const uint32_t r = pos + __popc(m & ((1u << (threadIdx.x & 31u)) - 1u));
+            sm.skey[r] = k;
+            sm.sidx[r] = x;
+        }
+        __syncthreads();
+    }
+    const uint32_t C = sm.misc[2];
+    const uint32_t P2 = next_pow2(C < 2 ? 2 : C);
+    for (uint32_t j = C + threadIdx.x; j < P2; j += blockDim.x) { sm.skey[j] = 0ull; sm.sidx[j] = NONE; }
+    bitonic_desc(sm.skey, sm.sidx, P2);
+    trace_mark(a, g, 2);
+    // merged rank of elite r: r + #(candidates with key > ekey[r]);
+    // of candidate j: j + #(elites with key >= ckey[j])  (elites win ties: lower index)
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+        const uint64_t k = sm.ekey[r];
+        uint32_t lo = 0, hi = C;
+        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.skey[mid] > k) lo = mid + 1; else hi = mid; }
+        const uint32_t rank = r + lo;
+        if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = r; }
+    }
+    for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
+        const uint64_t k = sm.skey[j];
+        uint32_t lo = 0, hi = E;
+        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.ekey[mid] >= k) lo = mid + 1; else hi = mid; }
+        const uint32_t rank = j + lo;
+        if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = sm.sidx[j]; }
+    }
+    __syncthreads();
+    leader_copy_elites(a, i, g, sm.okey, sm.oidx);
+    if (threadIdx.x == 0 && i == 0) a.ctl->n_fast = ++sm.misc[8];
+    trace_mark(a, g, 3);
+}
+
 // ------------------------------------------------------------------------
-// Breed (a4-a7 + fused a2) for one pair of children of island i.
+// Breed (a4-a7 + fused a2)
 // ------------------------------------------------------------------------
 template <int WT>
 __device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, uint32_t g, const double* fit)
@@ -969,33 +1241,49 @@ __device__ __forceinline__ void init_row(const GaArgs& a, Row<WT>& row, uint32_t
     }
 }
 
+
 // One child per thread.  The two children of a pair (c0 = E + 2q, c1 = c0 + 1)
 // sit in adjacent lanes and swap their tournament winners with one shuffle;
-// each lane then builds only its own child (R8, R18).
+// each lane then builds only its own child (R8, R18).  32-child chunks are
+// dealt round-robin over every worker warp of the island (warp-major), so all
+// SMs get the same share.
 template <int WT>
-__device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl, uint32_t cpi,
+__device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl,
                                                const uint64_t* popc, const double* fitc, uint64_t* popn,
-                                               double* fitn, const uint32_t* sP, const uint32_t* sO, uint64_t tau,
-                                               uint32_t* ccnt, uint64_t* ckey, uint32_t* cidx, BestRow<WT>& best)
+                                               double* fitn, const uint32_t* sP, const uint32_t* sO,
+                                               const uint64_t* tau_ptr, uint32_t* ccnt, uint64_t* ckey,
+                                               uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx, uint32_t snap)
 {
     const ChainDev& ch = a.ch;
     const uint32_t W = ch.W, N = a.N, E = a.E;
     const uint32_t nchild = N - E;
-    const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t stride = cpi * blockDim.x;
-    for (uint32_t base = wl * blockDim.x + (threadIdx.x & ~31u); base < nchild; base += stride) {
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const uint32_t chunks = (nchild + 31u) / 32u;
+    // snapshot of an earlier record of this island (a lower bound of the current one):
+    // only children that beat it can change the record (a8)
+    const double snap_f = __ldcg(a.snap_f + snap);
+    Row<WT> snap_r;
+#pragma unroll
+    for (int w = 0; w < WT; ++w)
+        snap_r.w[w] = (WT <= 16 && w < (int)W) ? __ldcg(a.snap_bits + (size_t)snap * W + w) : 0ull;
+    for (uint32_t cidx_ = warp * a.cpi + wl; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
+        const uint32_t base = cidx_ * 32u;
         const uint32_t t = base + lane;
         const bool valid = t < nchild;
         const uint32_t h = t & 1u;
         const uint32_t slot = E + t;
         const uint32_t gid = (a.island_base + i) * N + slot;
+        const bool tr = a.trace && threadIdx.x == 0 && blockIdx.x == a.I && g - a.g_begin < a.trace_gens &&
+                        cidx_ == wl;
         const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc) : 0u;     // a4
         const uint32_t other = __shfl_xor_sync(0xFFFFFFFFu, mine, 1);
+        if (tr) a.trace[(g - a.g_begin) * 16 + 8] = gtimer() + 0 * mine;
         if (!valid) continue;
         // first parent (positions < x) = own winner; second = the partner's
         Row<WT> A, B;
         row_load(A, popc + (size_t)mine * W, W);
         row_load(B, popc + (size_t)other * W, W);
+        if (tr) a.trace[(g - a.g_begin) * 16 + 9] = gtimer() + 0 * (A.w[0] ^ B.w[0]);
         const uint4 rx = philox10(make_uint4(gid - h, g, TAG_XOVER, 0), a.key0, a.key1);   // a5
         if ((uint64_t)rx.x < a.thr_c && ch.n >= 3) {
             const uint32_t x = 1 + below(rx.y, ch.n - 2);
@@ -1009,104 +1297,26 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);     // a6
         if ((uint64_t)rm.x < a.thr_m) row_xor_bit(A, below(rm.y, ch.n - 1));
         repair(a, A, gid, g);                                                              // a7
+        if (tr) a.trace[(g - a.g_begin) * 16 + 10] = gtimer() + 0 * A.w[0];
         const double f = eval_regs(ch, sP, sO, A, nullptr);                               // a2
+        if (tr) a.trace[(g - a.g_begin) * 16 + 11] = gtimer() + 0 * (uint64_t)__double_as_longlong(f);
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
-        append_if(fkey(f) > tau, ccnt, ckey, cidx, fkey(f), slot);
-        track_row(best, f, slot, A, W);
-    }
-}
-
-// Leader CTA of island i in the phase of generation g: record + stall of
-// generation g (a8), elites of generation g into slots 0..E-1 of g+1 (a3),
-// worst-elite key tau of generation g, reset of the candidate list that the
-// breed of the NEXT phase appends to.
-template <int WT>
-__device__ void leader_phase(const GaArgs& a, uint32_t i, uint32_t g, bool general, uint32_t cpi, const Smem& sm)
-{
-    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I;
-    const uint32_t cur = g & 1u, nxt = cur ^ 1u;
-    const uint32_t Lc = g % 3u, Lr = (g + 2u) % 3u;
-    trace_mark(a, g, 0);
-    leader_record<WT>(a, i, g, cur, cpi, sm);
-    trace_mark(a, g, 1);
-    const uint64_t* popc = a.pop[cur] + (size_t)i * N * W;
-    const double* fitc = a.fit[cur] + (size_t)i * N;
-    if (E > 0) {
-        if (general) {
-            leader_sort_selected(a, i, E, false, sm);
-        } else {
-            // previous elites (slots 0..E-1, ranked) merged with the candidates that
-            // beat the worst of them; the candidate list is a superset (lagged tau)
-            for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) sm.ekey[r] = fkey(__ldcg(fitc + r));
-            __syncthreads();
-            const uint64_t thr = sm.ekey[E - 1];
-            const uint32_t C0 = __ldcg(&a.cand_cnt[Lc * I + i]);
-            const uint64_t* ck = a.cand_key[Lc] + (size_t)i * N;
-            const uint32_t* cx = a.cand_idx[Lc] + (size_t)i * N;
-            // stable compaction of the useful candidates (key > worst elite) into smem
-            uint32_t* s_cnt = (uint32_t*)sm.scratch;     // scratch reused: 33 BestRef >= 9 u32
-            if (threadIdx.x == 0) s_cnt[0] = 0;
-            __syncthreads();
-            for (uint32_t j0 = 0; j0 < C0; j0 += blockDim.x) {
-                const uint32_t j = j0 + threadIdx.x;
-                uint64_t k = 0;
-                uint32_t x = NONE;
-                bool keep = false;
-                if (j < C0) { k = __ldcg(ck + j); x = __ldcg(cx + j); keep = k > thr; }
-                const unsigned m = __ballot_sync(0xFFFFFFFFu, keep);
-                uint32_t pos = 0;
-                if ((threadIdx.x & 31u) == 0 && m) pos = atomicAdd(&s_cnt[0], (uint32_t)__popc(m));
-                pos = __shfl_sync(0xFFFFFFFFu, pos, 0);
-                if (keep) {
-                    const uint32_t r = pos + __popc(m & ((1u << (threadIdx.x & 31u)) - 1u));
-                    sm.skey[r] = k;
-                    sm.sidx[r] = x;
-                }
+        append_if(fkey(f) > __ldcg(tau_ptr), ccnt, ckey, cidx, fkey(f), slot);
+        if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
+        bool improves = f > snap_f;
+        if (f == snap_f) {
+            if (WT > 16) {
+                improves = true;                      // wide rows: let the leader compare bits
+            } else {
+                bool decided = false;
+#pragma unroll
+                for (int w = WT - 1; w >= 0; --w)
+                    if (w < (int)W && !decided && A.w[w] != snap_r.w[w]) { improves = A.w[w] < snap_r.w[w]; decided = true; }
             }
-            __syncthreads();
-            const uint32_t C = s_cnt[0];
-            const uint32_t P2 = next_pow2(C < 2 ? 2 : C);
-            for (uint32_t j = C + threadIdx.x; j < P2; j += blockDim.x) { sm.skey[j] = 0ull; sm.sidx[j] = NONE; }
-            bitonic_desc(sm.skey, sm.sidx, P2);
-            trace_mark(a, g, 2);
-            // merged rank of elite r: r + #(candidates with key > ekey[r]);
-            // of candidate j: j + #(elites with key >= ckey[j])  (elites win ties: lower index)
-            for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
-                const uint64_t k = sm.ekey[r];
-                uint32_t lo = 0, hi = C;    // first j with skey[j] <= k
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.skey[mid] > k) lo = mid + 1; else hi = mid; }
-                const uint32_t rank = r + lo;
-                if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = r; }
-            }
-            for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
-                const uint64_t k = sm.skey[j];
-                uint32_t lo = 0, hi = E;    // first r with ekey[r] < k
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (sm.ekey[mid] >= k) lo = mid + 1; else hi = mid; }
-                const uint32_t rank = j + lo;
-                if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = sm.sidx[j]; }
-            }
-            __syncthreads();
         }
-        // copy the elites in rank order to slots 0..E-1 of generation g+1 (R18)
-        const uint64_t* rk = general ? sm.skey : sm.okey;
-        const uint32_t* rx = general ? sm.sidx : sm.oidx;
-        uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
-        double* fitn = a.fit[nxt] + (size_t)i * N;
-        for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
-            const uint32_t r = j / W, w = j % W;
-            popn[(size_t)r * W + w] = __ldcg(popc + (size_t)rx[r] * W + w);
-        }
-        for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(rk[r]);
-        if (threadIdx.x == 0) a.tau[cur * I + i] = rk[E - 1];
-    } else if (threadIdx.x == 0) {
-        a.tau[cur * I + i] = ~0ull;    // no elites: no candidate list
+        append_if(improves, rcnt, nullptr, ridx, 0, slot);
     }
-    if (threadIdx.x == 0) {
-        a.cand_cnt[Lr * I + i] = 0;
-        if (i == 0) { if (general) a.ctl->n_general++; else a.ctl->n_fast++; }
-    }
-    trace_mark(a, g, 3);
 }
 
 // ------------------------------------------------------------------------
@@ -1116,7 +1326,7 @@ __device__ void leader_phase(const GaArgs& a, uint32_t i, uint32_t g, bool gener
 // needs only generation g and a lagged candidate threshold.
 // ------------------------------------------------------------------------
 template <int WT>
-__global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
+__global__ void __launch_bounds__(kBlock, (WT <= 8 ? 3 : (WT <= 16 ? 2 : 1))) ga_kernel(GaArgs a)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     Smem sm;
@@ -1125,8 +1335,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
     stage_chain(sm.chain, a.ch, sm.mbar);
     const uint32_t* sP = sm.chain;
     const uint32_t* sO = sm.chain + a.ch.p_words;
-    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I;
-    const uint32_t cpi = (gridDim.x - I) / I;           // worker CTAs per island
+    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I, Ns = a.Ns, cpi = a.cpi, cpp = a.cpi_pad;
     const bool is_leader = blockIdx.x < I;
     const uint32_t widx = is_leader ? 0u : blockIdx.x - I;
     const uint32_t my_island = is_leader ? NONE : widx / cpi;
@@ -1138,11 +1347,14 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
         if (worker) {
             const uint32_t i = my_island;
             uint64_t* pop = a.pop[0] + (size_t)i * N * W;
-            double* fit = a.fit[0] + (size_t)i * N;
+            double* fit = a.fit[0] + (size_t)i * Ns;
             BestRow<WT> best;
             best.f = -CUDART_INF;
             best.idx = NONE;
-            for (uint32_t c = my_local * blockDim.x + threadIdx.x; c < N; c += cpi * blockDim.x) {
+            const uint32_t warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5, chunks = (N + 31u) / 32u;
+            for (uint32_t cc = warp * cpi + my_local; cc < chunks; cc += nwarps * cpi) {
+                const uint32_t c = cc * 32u + (threadIdx.x & 31u);
+                if (c >= N) continue;
                 Row<WT> r;
                 init_row(a, r, (a.island_base + i) * N + c);
                 const double f = eval_regs(a.ch, sP, sO, r, nullptr);
@@ -1151,7 +1363,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
                 track_row(best, f, c, r, W);
             }
             best = block_best_row(best, W, (BestRow<WT>*)sm.scratch);
-            if (threadIdx.x == 0) write_partial(a, (size_t)i * cpi + my_local, best, W);
+            if (threadIdx.x == 0) write_partial(a, (size_t)i * cpp + my_local, best, W);
         }
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             a.ctl->full = 1;
@@ -1159,9 +1371,14 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
             a.ctl->gens_run = 0;
             a.ctl->n_general = 0;
             a.ctl->n_fast = 0;
+            a.ctl->redo[0] = 0;
+            a.ctl->redo[1] = 0;
         }
         grid.sync();
-        if (is_leader) leader_record<WT>(a, blockIdx.x, 0, 0, cpi, sm);
+        if (is_leader) {
+            rec_load(a, blockIdx.x, sm);
+            leader_record<WT>(a, blockIdx.x, 0, 0, sm);
+        }
         return;
     }
 
@@ -1173,7 +1390,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
             const uint32_t i = blockIdx.x;
             leader_sort_selected(a, i, a.K, worst, sm);
             uint64_t* pop = a.pop[cur] + (size_t)i * N * W;
-            double* fit = a.fit[cur] + (size_t)i * N;
+            double* fit = a.fit[cur] + (size_t)i * Ns;
             if (!worst) {
                 // export the island's top-K (rows + fitness) to its slot of the gather buffer
                 const size_t gi = a.island_base + i;
@@ -1230,7 +1447,7 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
                 }
                 // the children's partial bests of this generation may point at replaced slots
                 for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x)
-                    a.part_idx[((size_t)cur * I + i) * cpi + j] = NONE;
+                    a.part_idx[((size_t)cur * I + i) * cpp + j] = NONE;
                 if (threadIdx.x == 0 && i == 0) a.ctl->full = 1;
             }
         }
@@ -1241,55 +1458,74 @@ __global__ void __launch_bounds__(kBlock) ga_kernel(GaArgs a)
     // list g%3 holds the candidates of generation g (consumed by leader(g)),
     // breed(g) appends generation g+1's to list (g+1)%3, leader(g) resets (g+2)%3.
     const bool first_full = __ldcg(&a.ctl->full) != 0;
+    uint32_t mph = 0;
+    if (is_leader) {
+        rec_load(a, blockIdx.x, sm);
+        if (threadIdx.x == 0) {
+            mbar_init(sm.mbar + 1, 1);
+            sm.misc[8] = __ldcg(&a.ctl->n_fast);
+            sm.misc[9] = __ldcg(&a.ctl->n_general);
+        }
+        __syncthreads();
+    }
     uint32_t g = a.g_begin;
     for (; g < a.g_end; ++g) {
         const uint32_t cur = g & 1u, nxt = cur ^ 1u;
-        const uint32_t Lc = g % 3u, Lb = (g + 1u) % 3u;
-        bool general = (g == a.g_begin) && first_full;
-        if (!general)
-            for (uint32_t i = 0; i < I; ++i) general |= __ldcg(&a.cand_cnt[Lc * I + i]) > kCandCap;
-        general = general && E > 0;
+        const uint32_t Lb = (g + 1u) % 3u;
         uint32_t tau_par = nxt;               // fast path: worst elite of generation g-1 (lagged)
-        if (general) {
+        if (g == a.g_begin && first_full && E > 0) {
+            // generation 0 or just after migration: exact top-E first, then breed
             general_select(a, a.fit[cur], E, false, sm, grid);
-            if (is_leader) leader_phase<WT>(a, blockIdx.x, g, true, cpi, sm);
+            if (is_leader) {
+                // the record of generation g_begin was taken by INIT or at the end of
+                // the previous segment (and by the migrant import)
+                leader_general(a, blockIdx.x, g, sm);
+                if (threadIdx.x == 0) {
+                    a.cand_cnt[((g + 2u) % 3u) * I + blockIdx.x] = 0;
+                    a.rc_cnt[((g + 2u) % 3u) * I + blockIdx.x] = 0;
+                    if (blockIdx.x == 0) a.ctl->n_general = ++sm.misc[9];
+                }
+            }
             grid.sync();
             if (__ldcg(&a.ctl->done)) break;
             tau_par = cur;                    // exact threshold of generation g
         } else if (is_leader) {
-            leader_phase<WT>(a, blockIdx.x, g, false, cpi, sm);
+            leader_fast<WT>(a, blockIdx.x, g, sm, mph);
         }
         if (worker) {
             // a4-a7 + a2: children of generation g+1
             const uint32_t i = my_island;
             if (threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
-                a.trace[(g - a.g_begin) * 8 + 4] = gtimer();
-            BestRow<WT> best;
-            best.f = -CUDART_INF;
-            best.idx = NONE;
-            uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
-            breed_children<WT>(a, i, g, my_local, cpi, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * N,
-                               popn, a.fit[nxt] + (size_t)i * N, sP, sO, __ldcg(&a.tau[tau_par * I + i]),
-                               a.cand_cnt + Lb * I + i, a.cand_key[Lb] + (size_t)i * N,
-                               a.cand_idx[Lb] + (size_t)i * N, best);
-            best = block_best_row(best, W, (BestRow<WT>*)sm.scratch);
-            if (threadIdx.x == 0) {
-                write_partial(a, ((size_t)nxt * I + i) * cpi + my_local, best, W);
-                if (blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
-                    a.trace[(g - a.g_begin) * 8 + 5] = gtimer();
-            }
+                a.trace[(g - a.g_begin) * 16 + 4] = gtimer();
+            breed_children<WT>(a, i, g, my_local, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * Ns,
+                               a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
+                               a.tau + tau_par * I + i, a.cand_cnt + Lb * I + i, a.cand_key[Lb] + (size_t)i * Ns,
+                               a.cand_idx[Lb] + (size_t)i * Ns, a.rc_cnt + Lb * I + i,
+                               a.rc_idx[Lb] + (size_t)i * Ns, nxt * I + i);
+            if (threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
+                a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
         }
         grid.sync();
         if (threadIdx.x == 0 && a.trace && g - a.g_begin < a.trace_gens) {
-            if (blockIdx.x == 0) a.trace[(g - a.g_begin) * 8 + 6] = gtimer();
-            if (blockIdx.x == I) a.trace[(g - a.g_begin) * 8 + 7] = gtimer();
+            if (blockIdx.x == 0) a.trace[(g - a.g_begin) * 16 + 6] = gtimer();
+            if (blockIdx.x == I) a.trace[(g - a.g_begin) * 16 + 7] = gtimer();
         }
-        if (g == a.g_begin && blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;   // all CTAs read it before this barrier
+        if (g == a.g_begin && blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;   // every CTA read it earlier
         if (__ldcg(&a.ctl->done)) break;
+        if (__ldcg(&a.ctl->redo[cur]) == g + 1) {
+            // a candidate list overflowed: exact top-E of generation g (still intact)
+            general_select(a, a.fit[cur], E, false, sm, grid);
+            if (is_leader) {
+                leader_general(a, blockIdx.x, g, sm);
+                if (threadIdx.x == 0 && blockIdx.x == 0) a.ctl->n_general = ++sm.misc[9];
+            }
+            grid.sync();
+        }
     }
-    if (g == a.g_end) {
+    if (g == a.g_end && is_leader) {
         // record (and stall) of the last generation of the segment
-        if (is_leader) leader_record<WT>(a, blockIdx.x, g, g & 1u, cpi, sm);
+        const uint32_t R = __ldcg(a.rc_cnt + (g % 3u) * I + blockIdx.x);
+        leader_record_list<WT>(a, blockIdx.x, g, R, false, sm);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->gens_run = g;
 }
@@ -1394,6 +1630,12 @@ static void* ga_pick(uint32_t W)
     return ga_fn<64>();
 }
 
+int ga_max_blocks_per_sm(uint32_t W)
+{
+    const uint32_t wt = wt_of(W);
+    return wt <= 8 ? 3 : (wt <= 16 ? 2 : 1);
+}
+
 int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err)
 {
     void* fn = ga_pick(a.ch.W);
@@ -1406,12 +1648,10 @@ int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err)
     return per_sm * num_sms;
 }
 
-cudaError_t launch_ga(const GaArgs& a, cudaStream_t st, int num_sms, uint64_t* launches)
+cudaError_t launch_ga(const GaArgs& a, int grid, cudaStream_t st, uint64_t* launches)
 {
     cudaError_t e;
-    const int grid = ga_grid(a, num_sms, &e);
-    if (e != cudaSuccess) return e;
-    if (grid < (int)a.I) return cudaErrorInvalidConfiguration;
+    if (grid < 2 * (int)a.I) return cudaErrorInvalidConfiguration;
     void* fn = ga_pick(a.ch.W);
     GaArgs copy = a;
     void* args[] = {&copy};
