@@ -1259,13 +1259,6 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
     const uint32_t nchild = N - E;
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const uint32_t chunks = (nchild + 31u) / 32u;
-    // snapshot of an earlier record of this island (a lower bound of the current one):
-    // only children that beat it can change the record (a8)
-    const double snap_f = __ldcg(a.snap_f + snap);
-    Row<WT> snap_r;
-#pragma unroll
-    for (int w = 0; w < WT; ++w)
-        snap_r.w[w] = (WT <= 16 && w < (int)W) ? __ldcg(a.snap_bits + (size_t)snap * W + w) : 0ull;
     for (uint32_t cidx_ = warp * a.cpi + wl; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
         const uint32_t base = cidx_ * 32u;
         const uint32_t t = base + lane;
@@ -1304,6 +1297,9 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         fitn[slot] = f;
         append_if(fkey(f) > __ldcg(tau_ptr), ccnt, ckey, cidx, fkey(f), slot);
         if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
+        // a8 filter: only children that beat a snapshot of an earlier record of this
+        // island (a lower bound of the current record) can change the record
+        const double snap_f = __ldcg(a.snap_f + snap);
         bool improves = f > snap_f;
         if (f == snap_f) {
             if (WT > 16) {
@@ -1311,8 +1307,12 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
             } else {
                 bool decided = false;
 #pragma unroll
-                for (int w = WT - 1; w >= 0; --w)
-                    if (w < (int)W && !decided && A.w[w] != snap_r.w[w]) { improves = A.w[w] < snap_r.w[w]; decided = true; }
+                for (int w = WT - 1; w >= 0; --w) {
+                    if (w < (int)W && !decided) {
+                        const uint64_t sw = __ldcg(a.snap_bits + (size_t)snap * W + w);
+                        if (A.w[w] != sw) { improves = A.w[w] < sw; decided = true; }
+                    }
+                }
             }
         }
         append_if(improves, rcnt, nullptr, ridx, 0, slot);
