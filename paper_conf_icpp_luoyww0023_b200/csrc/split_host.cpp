@@ -332,7 +332,26 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
             return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
         }
     }
+    // interleaved {P[p+1], ovh[p]} table for the eval kernel's walk
+    const uint32_t po_n = ((n - 1) + 1) & ~1u;                  // entries, even -> 16-byte multiple
+    std::vector<uint32_t> po(2 * (size_t)po_n, 0);
+    for (uint32_t q = 0; q + 1 < n; ++q) {
+        po[2 * q] = words[q + 1];
+        po[2 * q + 1] = (uint32_t)ovh[q];
+    }
+    uint32_t* d_po = nullptr;
+    TRY(dalloc(h, &d_po, po.size()));
+    {
+        cudaError_t e = cudaMemcpy(d_po, po.data(), po.size() * 4, cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) {
+            free_all(h);
+            delete h;
+            return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
+        }
+    }
     ChainDev& ch = h->ch;
+    ch.po = (const uint2*)d_po;
+    ch.po_bytes = (uint32_t)(po.size() * 4);
     ch.words = d_chain;
     ch.n = n;
     ch.W = h->W;

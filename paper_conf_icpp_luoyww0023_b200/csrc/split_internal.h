@@ -36,6 +36,8 @@ struct ChainDev {
     uint32_t T;                 // == P[n]
     uint32_t k_min, k_max;
     uint64_t last_mask;         // valid bits of word W-1
+    const uint2* po;            // device: po[p] = {P[p+1], ovh[p]}, p in [0, n-2] (padded)
+    uint32_t po_bytes;          // multiple of 16
 };
 
 // All device pointers and scalars the GA kernel needs (passed by value).

@@ -182,6 +182,76 @@ __device__ __forceinline__ void stage_chain(uint32_t* s_chain, const ChainDev& c
     }
 }
 
+// ------------------------------------------------------------------------
+// mbarrier + TMA bulk copies (cp.async.bulk) for the leader's loads
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* mbar, uint32_t bytes)
+{
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* mbar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t parity)
+{
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(ok)
+            : "r"(smem_u32(mbar)), "r"(parity)
+            : "memory");
+    }
+}
+// bytes: multiple of 16; src/dst 16-byte aligned
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* mbar)
+{
+    const uint32_t d = smem_u32(dst), b = smem_u32(mbar);
+    for (uint32_t off = 0; off < bytes; off += 32768u) {
+        const uint32_t n = (bytes - off < 32768u) ? (bytes - off) : 32768u;
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d + off),
+                     "l"((const char*)src + off), "r"(n), "r"(b)
+                     : "memory");
+    }
+}
+// Stage `bytes` (multiple of 16) of global memory into shared memory with TMA
+// bulk copies completing on one mbarrier; all threads return after arrival.
+__device__ __forceinline__ void stage_bulk(void* s_dst, const void* src, uint32_t bytes, uint64_t* mbar)
+{
+    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(s_dst);
+        for (uint32_t off = 0; off < bytes; off += 32768u) {
+            const uint32_t b = (bytes - off < 32768u) ? (bytes - off) : 32768u;
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst + off),
+                "l"((const char*)src + off), "r"(b), "r"(bar)
+                : "memory");
+        }
+    }
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+            : "=r"(ok)
+            : "r"(bar)
+            : "memory");
+    }
+}
+
 // Walk the cuts of one candidate: words come from `get(w)` in ascending order.
 // Block j ends at cut c_j; t_j = P[c_j+1] - P[c_{j-1}+1] + ovh[c_{j-1}] (R3).
 struct Stats {
@@ -287,58 +357,79 @@ __global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_kernel(ChainDev ch
 // handled as 2W 32-bit half-words and each lane keeps a bitmask of its
 // non-empty half-words, so the walk takes exactly one iteration per cut
 // (no per-word loop whose trip count diverges across the warp).
+// K1 for W <= 16.  Each warp streams 32-row tiles (32*W u64, contiguous) into
+// a double-buffered shared tile with TMA bulk copies (cp.async.bulk + one
+// mbarrier per buffer), so no instructions are spent staging.  Lane l owns row
+// l: a skewed pass (lane l reads half-word (q+l)%H at step q: conflict-free)
+// counts cuts and builds a bitmask of non-empty half-words, then the walk takes
+// exactly one iteration per cut.
 template <int W>
 __global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
                                                                        uint64_t n_cand, double* __restrict__ out)
 {
     constexpr uint32_t H = 2 * W;          // 32-bit halves per row
-    constexpr uint32_t PITCH = H + 1;      // odd pitch: lanes read distinct banks
+    constexpr uint32_t TILE = 32 * H;      // u32 per tile
     extern __shared__ __align__(16) uint8_t smem[];
-    uint32_t* s_chain = (uint32_t*)smem;
-    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
-    uint32_t* s_tiles = (uint32_t*)(mbar + 2);
-    stage_chain(s_chain, ch, mbar);
-    const uint32_t* sP = s_chain;
-    const uint32_t* sO = s_chain + ch.p_words;
+    // staged chain: po[p] = {P[p+1], ovh[p]} for cut positions p in [0, n-2]
+    const uint2* spo = (const uint2*)smem;
+    uint64_t* mbar = (uint64_t*)(smem + ch.po_bytes);            // [0] chain, [1 + 2*warp + b] tiles
+    uint32_t* s_tiles = (uint32_t*)(mbar + 2 * kEvalWarps + 2);  // 16-byte aligned
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    uint32_t* tile = s_tiles + warp * 32u * PITCH;
-    // valid bits: positions [0, n-2] -> halves [0, qfull) full, half qfull partial
+    uint64_t* wbar = mbar + 2 + 2 * warp;
+    if (lane == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(wbar)));
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(wbar + 1)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    stage_bulk(smem, ch.po, ch.po_bytes, mbar);                   // includes a __syncthreads
+    uint32_t* tiles = s_tiles + warp * 2u * TILE;
     const uint32_t npos = ch.n - 1, qfull = npos >> 5;
     const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
+    const uint64_t n_full = n_cand / 32;                           // full tiles go through TMA
     const uint64_t n_tiles = (n_cand + 31) / 32;
     const uint64_t nw = (uint64_t)gridDim.x * kEvalWarps;
-    for (uint64_t t = (uint64_t)blockIdx.x * kEvalWarps + warp; t < n_tiles; t += nw) {
+    uint64_t t = (uint64_t)blockIdx.x * kEvalWarps + warp;
+    auto issue = [&](uint64_t tt, uint32_t b) {
+        if (lane == 0 && tt < n_full) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_expect_tx(wbar + b, TILE * 4u);
+            bulk_g2s(tiles + b * TILE, bits + tt * 32 * W, TILE * 4u, wbar + b);
+        }
+    };
+    issue(t, 0);
+    uint32_t ph = 0;                       // bit b: parity of buffer b's next phase
+    for (uint32_t b = 0; t < n_tiles; t += nw, b ^= 1u) {
+        issue(t + nw, b ^ 1u);
+        uint32_t* tile = tiles + b * TILE;
         const uint64_t row0 = t * 32;
         const uint32_t rows = (uint32_t)((n_cand - row0) < 32 ? (n_cand - row0) : 32);
-        if (rows == 32) {
-            const uint4* src4 = (const uint4*)(bits + row0 * W);   // 256*W bytes, 16-byte aligned
-#pragma unroll
-            for (uint32_t it = 0; it < (16 * W + 31) / 32; ++it) {
-                const uint32_t j = lane + 32 * it;
-                if (j < 16 * W) {
-                    const uint4 v = __ldcs(src4 + j);
-                    const uint32_t e = 4 * j;       // first half-word of the chunk; e and H are even
-                    const uint32_t r = e / H, c = e % H;
-                    uint32_t* d = tile + r * PITCH + c;
-                    d[0] = v.x; d[1] = v.y;
-                    if (c + 2 < H) { d[2] = v.z; d[3] = v.w; }
-                    else { d[PITCH - c] = v.z; d[PITCH - c + 1] = v.w; }   // c + 2 == H: row r+1, halves 0-1
-                }
-            }
+        if (t < n_full) {
+            mbar_wait(wbar + b, (ph >> b) & 1u);
+            ph ^= 1u << b;
         } else {
             const uint32_t* src = (const uint32_t*)(bits + row0 * W);
-            for (uint32_t e = lane; e < rows * H; e += 32) tile[(e / H) * PITCH + (e % H)] = __ldcs(src + e);
+            for (uint32_t e = lane; e < rows * H; e += 32) tile[e] = __ldcs(src + e);
+            __syncwarp();
         }
-        __syncwarp();
         if (lane < rows) {
-            const uint32_t* my = tile + lane * PITCH;
-            uint32_t cuts = 0, occ = 0;
+            uint32_t* my = tile + lane * H;
+            uint32_t cuts = 0, occr = 0;
 #pragma unroll
             for (uint32_t q = 0; q < H; ++q) {
-                uint32_t v = my[q];
-                v &= (q < qfull) ? ~0u : (q == qfull ? lastm : 0u);
+                const uint32_t v = my[(q + lane) % H];
                 cuts += __popc(v);
-                occ |= (v != 0u ? 1u : 0u) << q;
+                occr |= (v != 0u ? 1u : 0u) << q;
+            }
+            // bit q of occr is half (q + lane) % H: rotate into place
+            uint32_t occ = (H == 32) ? __funnelshift_l(occr, occr, lane)
+                                     : (((occr << (lane % H)) | (occr >> ((H - lane % H) % H))) & (H == 32 ? ~0u : ((1u << H) - 1u)));
+            // padding (positions >= n-1): only halves >= qfull, usually one
+            for (uint32_t q = qfull; q < H; ++q) {
+                const uint32_t v = my[q];
+                const uint32_t keep = (q == qfull) ? (v & lastm) : 0u;
+                cuts -= __popc(v ^ keep);
+                my[q] = keep;
+                if (!keep) occ &= ~(1u << q);
             }
             const uint32_t k = cuts + 1;
             double f = -CUDART_INF;
@@ -349,16 +440,16 @@ __global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_w_kernel(ChainDev 
                     if (v == 0u) {
                         q = __ffs(occ) - 1;
                         occ &= occ - 1;
-                        v = my[q] & ((q < qfull) ? ~0u : lastm);
+                        v = my[q];
                     }
                     const uint32_t p = 32u * q + (uint32_t)(__ffs(v) - 1);
                     v &= v - 1;
-                    const uint32_t Pp = sP[p + 1];
-                    const uint32_t tj = Pp - startP + prev_o;
+                    const uint2 e = spo[p];
+                    const uint32_t tj = e.x - startP + prev_o;
                     S2 += (uint64_t)tj * tj;
-                    prev_o = sO[p];
-                    OV += prev_o;
-                    startP = Pp;
+                    OV += e.y;
+                    startP = e.x;
+                    prev_o = e.y;
                 }
                 const uint32_t tl = ch.T - startP + prev_o;
                 S2 += (uint64_t)tl * tl;
@@ -727,45 +818,6 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     return off;
 }
 
-// ------------------------------------------------------------------------
-// mbarrier + TMA bulk copies (cp.async.bulk) for the leader's loads
-// ------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count)
-{
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count));
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* mbar, uint32_t bytes)
-{
-    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* mbar, uint32_t bytes)
-{
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t parity)
-{
-    uint32_t ok = 0;
-    while (!ok) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-            : "=r"(ok)
-            : "r"(smem_u32(mbar)), "r"(parity)
-            : "memory");
-    }
-}
-// bytes: multiple of 16; src/dst 16-byte aligned
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* mbar)
-{
-    const uint32_t d = smem_u32(dst), b = smem_u32(mbar);
-    for (uint32_t off = 0; off < bytes; off += 32768u) {
-        const uint32_t n = (bytes - off < 32768u) ? (bytes - off) : 32768u;
-        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d + off),
-                     "l"((const char*)src + off), "r"(n), "r"(b)
-                     : "memory");
-    }
-}
 __host__ __device__ inline uint32_t round16(uint32_t bytes) { return (bytes + 15u) & ~15u; }
 
 // composite of element i of an island: desc order (elite/export) -> (key, ~idx);
@@ -1567,8 +1619,8 @@ __global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
 // ------------------------------------------------------------------------
 static size_t eval_smem(const ChainDev& ch)
 {
-    const size_t tile = ch.W <= 16 ? (size_t)(2 * ch.W + 1) * 4 : (size_t)(ch.W | 1u) * 8;
-    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * tile;
+    if (ch.W <= 16) return (size_t)ch.po_bytes + 16 * (kEvalWarps + 1) + (size_t)kEvalWarps * 2 * 32 * (2 * ch.W) * 4;
+    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
 }
 
 template <int W>
