@@ -698,7 +698,7 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
         CU(cudaMemcpy(tr.data(), h->d_trace, tr.size() * 8, cudaMemcpyDeviceToHost));
         if (FILE* f = fopen(getenv("SPLIT_TRACE"), "w")) {
             fprintf(f, "gen,lead_start,lead_record,lead_sort,lead_end,work_start,work_end,lead_sync,work_sync,"
-                       "b_tourn,b_rows,b_repair,b_eval,b_store,w_loopend,w_allwarps,lead_loaded\n");
+                       "b_tourn,b_rows,b_repair,b_eval,b_rec,b_xover,b_cand,lead_loaded\n");
             CU(cudaMemset(h->d_trace, 0, tr.size() * 8));
             for (uint32_t g = 0; g < h->trace_gens; ++g) {
                 fprintf(f, "%u", g);

@@ -28,6 +28,11 @@ namespace cg = cooperative_groups;
 namespace splitga {
 
 constexpr uint32_t NONE = 0xFFFFFFFFu;
+#ifdef SPLIT_TRACE_BUILD
+constexpr bool kTrace = true;     // phase timestamps (tools: SPLIT_TRACE=<csv>)
+#else
+constexpr bool kTrace = false;
+#endif
 
 // ------------------------------------------------------------------------
 // Philox4x32-10 (Salmon et al., SC'11), multipliers/Weyl constants of the
@@ -75,7 +80,10 @@ __device__ __forceinline__ double dexp_dev(double z)
 {
     if (z > 710.0) return CUDART_INF;
     if (z < -700.0) return 0.0;
-    const double j = rint(__dmul_rn(z, 0x1.71547652b82fep+0));
+    // j = rint(z / ln 2), ties to even: adding 1.5*2^52 rounds to an integer (RN)
+    const double t = __dadd_rn(__dmul_rn(z, 0x1.71547652b82fep+0), 0x1.8p52);
+    const double j = __dsub_rn(t, 0x1.8p52);
+    const int ji = (int)(uint32_t)__double_as_longlong(t);     // low word of t holds j
     double r = __fma_rn(-j, 0x1.62e42fefa39efp-1, z);
     r = __fma_rn(-j, 0x1.abc9e3b39803fp-56, r);
     double p = 0x1.6124613a86d09p-33;           // 1/13!
@@ -92,7 +100,11 @@ __device__ __forceinline__ double dexp_dev(double z)
     p = __fma_rn(p, r, 0.5);
     p = __fma_rn(p, r, 1.0);
     p = __fma_rn(p, r, 1.0);
-    return ldexp(p, (int)j);
+    // ldexp(p, j) for j in [-2, 1024]: exact scaling by powers of two (p in [0.7, 1.5])
+    const int j1 = ji > 1023 ? 1023 : ji;
+    const double s1 = __longlong_as_double((long long)(j1 + 1023) << 52);
+    const double s2 = __longlong_as_double((long long)(ji - j1 + 1023) << 52);
+    return __dmul_rn(__dmul_rn(p, s1), s2);
 }
 
 // Eq. 2 from the exact integer statistics (R5'):
@@ -116,7 +128,7 @@ __device__ __forceinline__ unsigned long long gtimer()
 // after the generation barrier 6 (CTA 0) and 7 (last CTA)
 __device__ __forceinline__ void trace_mark(const GaArgs& a, uint32_t g, uint32_t slot)
 {
-    if (!a.trace || threadIdx.x != 0 || blockIdx.x != 0) return;
+    if (!kTrace || !a.trace || threadIdx.x != 0 || blockIdx.x != 0) return;
     const uint32_t gi = g - a.g_begin;
     if (gi < a.trace_gens) a.trace[gi * 16 + slot] = gtimer();
 }
@@ -553,16 +565,40 @@ template <int WT>
 __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
                                             const Row<WT>& r, Stats* st)
 {
-    return eval_walk(
-        ch, sP, sO,
-        [&](uint32_t w) {
-            uint64_t v = 0;
+    // same arithmetic as eval_walk, with the word loop unrolled over the register row
+    uint32_t cuts = 0;
 #pragma unroll
-            for (int i = 0; i < WT; ++i)
-                if ((uint32_t)i == w) v = r.w[i];
-            return v;
-        },
-        st);
+    for (int w = 0; w < WT; ++w)
+        if (w < (int)ch.W) cuts += __popcll(r.w[w] & word_mask(ch, w));
+    const uint32_t k = cuts + 1;
+    if (k < ch.k_min || k > ch.k_max) {
+        if (st) st->k = k;
+        return -CUDART_INF;
+    }
+    uint32_t startP = 0, prev_o = 0;
+    uint64_t S2 = 0, OV = 0;
+#pragma unroll
+    for (int w = 0; w < WT; ++w) {
+        if (w < (int)ch.W) {
+            uint64_t v = r.w[w] & word_mask(ch, w);
+            while (v) {
+                const uint32_t p = 64u * w + (uint32_t)(__ffsll((long long)v) - 1);
+                v &= v - 1;
+                const uint32_t Pp = sP[p + 1];
+                const uint32_t t = Pp - startP + prev_o;
+                S2 += (uint64_t)t * t;
+                prev_o = sO[p];
+                OV += prev_o;
+                startP = Pp;
+            }
+        }
+    }
+    const uint32_t t = ch.T - startP + prev_o;
+    S2 += (uint64_t)t * t;
+    const uint64_t S1 = (uint64_t)ch.T + OV;
+    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+    if (st) { st->k = k; st->V = V; st->S1 = S1; st->S2 = S2; st->OV = OV; }
+    return eq2(k, V, OV, ch.T);
 }
 
 // best-record order: (f desc, bitset asc; word W-1 most significant)
@@ -1168,7 +1204,7 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
     }
     mbar_wait(sm.mbar + 1, mph);
     mph ^= 1u;
-    if (a.trace && threadIdx.x == 0 && blockIdx.x == 0 && g - a.g_begin < a.trace_gens)
+    if (kTrace && a.trace && threadIdx.x == 0 && blockIdx.x == 0 && g - a.g_begin < a.trace_gens)
         a.trace[(g - a.g_begin) * 16 + 15] = gtimer();
     const uint32_t C0 = E > 0 ? sm.misc[4 + ((Lc * I + i) & 3u)] : 0u;
     const uint32_t R = sm.misc[16 + ((Lc * I + i) & 3u)];
@@ -1318,8 +1354,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         const uint32_t h = t & 1u;
         const uint32_t slot = E + t;
         const uint32_t gid = (a.island_base + i) * N + slot;
-        const bool tr = a.trace && threadIdx.x == 0 && blockIdx.x == a.I && g - a.g_begin < a.trace_gens &&
-                        cidx_ == wl;
+        const bool tr = kTrace && a.trace && threadIdx.x == 0 && blockIdx.x == a.I &&
+                        g - a.g_begin < a.trace_gens && cidx_ == wl;
         const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc) : 0u;     // a4
         const uint32_t other = __shfl_xor_sync(0xFFFFFFFFu, mine, 1);
         if (tr) a.trace[(g - a.g_begin) * 16 + 8] = gtimer() + 0 * mine;
@@ -1339,6 +1375,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
                 A.w[w] = (A.w[w] & m) | (B.w[w] & ~m);
             }
         }
+        if (tr) a.trace[(g - a.g_begin) * 16 + 13] = gtimer() + 0 * A.w[0];
         const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);     // a6
         if ((uint64_t)rm.x < a.thr_m) row_xor_bit(A, below(rm.y, ch.n - 1));
         repair(a, A, gid, g);                                                              // a7
@@ -1348,6 +1385,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
         append_if(fkey(f) > __ldcg(tau_ptr), ccnt, ckey, cidx, fkey(f), slot);
+        if (tr) a.trace[(g - a.g_begin) * 16 + 14] = gtimer();
         if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
         // a8 filter: only children that beat a snapshot of an earlier record of this
         // island (a lower bound of the current record) can change the record
@@ -1547,18 +1585,18 @@ __global__ void __launch_bounds__(kBlock, (WT <= 8 ? 3 : (WT <= 16 ? 2 : 1))) ga
         if (worker) {
             // a4-a7 + a2: children of generation g+1
             const uint32_t i = my_island;
-            if (threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
+            if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 4] = gtimer();
             breed_children<WT>(a, i, g, my_local, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * Ns,
                                a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
                                a.tau + tau_par * I + i, a.cand_cnt + Lb * I + i, a.cand_key[Lb] + (size_t)i * Ns,
                                a.cand_idx[Lb] + (size_t)i * Ns, a.rc_cnt + Lb * I + i,
                                a.rc_idx[Lb] + (size_t)i * Ns, nxt * I + i);
-            if (threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
+            if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
         }
         grid.sync();
-        if (threadIdx.x == 0 && a.trace && g - a.g_begin < a.trace_gens) {
+        if (kTrace && threadIdx.x == 0 && a.trace && g - a.g_begin < a.trace_gens) {
             if (blockIdx.x == 0) a.trace[(g - a.g_begin) * 16 + 6] = gtimer();
             if (blockIdx.x == I) a.trace[(g - a.g_begin) * 16 + 7] = gtimer();
         }
