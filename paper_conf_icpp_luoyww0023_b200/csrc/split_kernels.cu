@@ -1416,7 +1416,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
 // needs only generation g and a lagged candidate threshold.
 // ------------------------------------------------------------------------
 template <int WT>
-__global__ void __launch_bounds__(kBlock, (WT <= 8 ? 3 : (WT <= 16 ? 2 : 1))) ga_kernel(GaArgs a)
+__global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     Smem sm;
@@ -1722,8 +1722,8 @@ static void* ga_pick(uint32_t W)
 
 int ga_max_blocks_per_sm(uint32_t W)
 {
-    const uint32_t wt = wt_of(W);
-    return wt <= 8 ? 3 : (wt <= 16 ? 2 : 1);
+    (void)W;
+    return 1;
 }
 
 int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err)
