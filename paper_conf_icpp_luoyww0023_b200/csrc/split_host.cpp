@@ -414,11 +414,17 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
         TRY(dalloc(h, &a.pop[b], IN * h->W));
         TRY(dalloc(h, &a.fit[b], INs));
     }
-    for (int b = 0; b < 3; ++b) {
-        TRY(dalloc(h, &a.cand_key[b], INs));
-        TRY(dalloc(h, &a.cand_idx[b], INs));
+    {
+        // candidate regions: worker CTA c of an island produces at most 32 children per
+        // chunk it is dealt (chunks round-robin over cpi CTAs x warps)
+        const uint32_t chunks = (a.N - a.E + 31u) / 32u;
+        a.creg = 32u * ((chunks + a.cpi - 1u) / a.cpi) + 32u;
     }
-    TRY(dalloc(h, &a.cand_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4));   // 16-byte chunks readable
+    for (int b = 0; b < 3; ++b) {
+        TRY(dalloc(h, &a.cand_key[b], (size_t)a.I * a.cpi * a.creg));
+        TRY(dalloc(h, &a.cand_idx[b], (size_t)a.I * a.cpi * a.creg));
+    }
+    TRY(dalloc(h, &a.cand_cnt, 3 * (size_t)a.I * a.cpi_pad));
     TRY(dalloc(h, &a.rc_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4));
     for (int b = 0; b < 3; ++b) TRY(dalloc(h, &a.rc_idx[b], INs));
     TRY(dalloc(h, &a.snap_f, 2 * (size_t)a.I));
@@ -605,7 +611,7 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     a.stall_in_kernel = single ? 1u : 0u;
     h->stats = split_run_stats{};
     CU(cudaMemsetAsync(a.rec_valid, 0, a.I * 4, h->stream));
-    CU(cudaMemsetAsync(a.cand_cnt, 0, 3 * a.I * 4, h->stream));
+    CU(cudaMemsetAsync(a.cand_cnt, 0, 3 * (size_t)a.I * a.cpi_pad * 4, h->stream));
     CU(cudaMemsetAsync(a.rc_cnt, 0, 3 * a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.sel_cnt, 0, a.I * 4, h->stream));
     CU(cudaMemsetAsync(a.ghist, 0, 3 * a.I * 256 * 4, h->stream));

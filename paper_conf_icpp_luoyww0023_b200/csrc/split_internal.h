@@ -56,9 +56,10 @@ struct GaArgs {
     uint32_t stage_bits;               // leader stages partial bits in smem (small W)
     uint64_t* pop[2];                  // [I][N][W]
     double* fit[2];                    // [I][Ns]
-    uint64_t* cand_key[3];             // [I][Ns]  candidates of generation g (list g%3)
-    uint32_t* cand_idx[3];
-    uint32_t* cand_cnt;                // [3][I]
+    uint64_t* cand_key[3];             // [I][cpi][creg] candidates of generation g (list g%3),
+    uint32_t* cand_idx[3];             //   one region per worker CTA
+    uint32_t* cand_cnt;                // [3][I][cpi_pad] per-CTA candidate counts
+    uint32_t creg;                     // region size per worker CTA
     uint64_t* sel_key;                 // [I][kMaxElite] general-select / elite output
     uint32_t* sel_idx;
     uint32_t* sel_cnt;                 // [I]

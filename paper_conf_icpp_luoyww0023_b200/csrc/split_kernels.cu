@@ -849,7 +849,7 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take((size_t)kMaxElite * 4); if (s) s->oidx = (uint32_t*)p;
     p = take(sizeof(RecCache) + 8 * (size_t)a.ch.W); if (s) s->rec = (RecCache*)p;
     p = take((size_t)a.cpi_pad * 8); if (s) s->pf = (double*)p;
-    p = take((size_t)a.cpi_pad * 4); if (s) s->pi = (uint32_t*)p;
+    p = take(((size_t)a.cpi_pad + 4) * 4); if (s) s->pi = (uint32_t*)p;
     p = take(a.stage_bits ? (size_t)a.cpi_pad * a.ch.W * 8 : 16); if (s) s->pb = (uint64_t*)p;
     return off;
 }
@@ -1189,30 +1189,63 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
         // one TMA batch: record-candidate count (its 16-byte chunk) + a window of the
         // list, previous elites' fitness, candidate count chunk + a window of the list
         const uint32_t cnt_off = Lc * I + i;
-        const uint32_t win = Ns < kCandCap ? Ns : kCandCap;      // Ns is a multiple of 4
         const uint32_t rwin = Ns < kRecWin ? Ns : kRecWin;
-        const uint32_t b = 16u + rwin * 4u + (E > 0 ? round16(E * 8u) + 16u + win * 12u : 0u);
+        const uint32_t b = 16u + rwin * 4u + (E > 0 ? round16(E * 8u) + cpp * 4u : 0u);
         mbar_arrive_expect_tx(sm.mbar + 1, b);
         bulk_g2s(sm.misc + 16, a.rc_cnt + (cnt_off & ~3u), 16u, sm.mbar + 1);
         bulk_g2s(sm.rcw, a.rc_idx[Lc] + (size_t)i * Ns, rwin * 4u, sm.mbar + 1);
         if (E > 0) {
             bulk_g2s(sm.ekey, a.fit[cur] + (size_t)i * Ns, round16(E * 8u), sm.mbar + 1);
-            bulk_g2s(sm.misc + 4, a.cand_cnt + (cnt_off & ~3u), 16u, sm.mbar + 1);
-            bulk_g2s(sm.skey, a.cand_key[Lc] + (size_t)i * Ns, win * 8u, sm.mbar + 1);
-            bulk_g2s(sm.sidx, a.cand_idx[Lc] + (size_t)i * Ns, win * 4u, sm.mbar + 1);
+            bulk_g2s(sm.pi, a.cand_cnt + ((size_t)Lc * I + i) * cpp, cpp * 4u, sm.mbar + 1);   // per-CTA counts
         }
     }
     mbar_wait(sm.mbar + 1, mph);
     mph ^= 1u;
     if (kTrace && a.trace && threadIdx.x == 0 && blockIdx.x == 0 && g - a.g_begin < a.trace_gens)
         a.trace[(g - a.g_begin) * 16 + 15] = gtimer();
-    const uint32_t C0 = E > 0 ? sm.misc[4 + ((Lc * I + i) & 3u)] : 0u;
     const uint32_t R = sm.misc[16 + ((Lc * I + i) & 3u)];
+    uint32_t C0 = 0;
+    if (E > 0) {
+        // exclusive prefix of the per-CTA candidate counts (in place), total in misc[3]
+        uint32_t* cnt = sm.pi;
+        if (threadIdx.x < 32) {
+            uint32_t carry = 0;
+            for (uint32_t c0 = 0; c0 < cpi; c0 += 32) {
+                const uint32_t c = c0 + threadIdx.x;
+                const uint32_t v = c < cpi ? cnt[c] : 0u;
+                uint32_t incl = v;
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, incl, off);
+                    if (threadIdx.x >= (uint32_t)off) incl += o;
+                }
+                if (c < cpi) cnt[c] = carry + incl - v;
+                carry += __shfl_sync(0xFFFFFFFFu, incl, 31);
+            }
+            if (threadIdx.x == 0) { sm.misc[3] = carry; cnt[cpi] = carry; }
+        }
+        __syncthreads();
+        C0 = sm.misc[3];
+        if (C0 <= kCandCap) {
+            // gather every region into skey/sidx: warp w takes regions w, w+16, ...
+            const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+            const uint64_t* ck = a.cand_key[Lc] + (size_t)i * cpi * a.creg;
+            const uint32_t* cx = a.cand_idx[Lc] + (size_t)i * cpi * a.creg;
+            for (uint32_t c = warp; c < cpi; c += nwarps) {
+                const uint32_t o = cnt[c], nc = cnt[c + 1] - o;
+                for (uint32_t j = lane; j < nc; j += 32) {
+                    sm.skey[o + j] = __ldcg(ck + (size_t)c * a.creg + j);
+                    sm.sidx[o + j] = __ldcg(cx + (size_t)c * a.creg + j);
+                }
+            }
+        }
+        __syncthreads();
+    }
     const bool ok = C0 <= kCandCap;
     // a8: record of generation g
     leader_record_list<WT>(a, i, g, R, true, sm);
     trace_mark(a, g, 1);
-    if (threadIdx.x == 0) { a.cand_cnt[Lr * I + i] = 0; a.rc_cnt[Lr * I + i] = 0; }
+    if (threadIdx.x == 0) a.rc_cnt[Lr * I + i] = 0;
     if (E == 0) {
         if (threadIdx.x == 0) a.tau[cur * I + i] = ~0ull;
         return;
@@ -1274,12 +1307,13 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
 // Breed (a4-a7 + fused a2)
 // ------------------------------------------------------------------------
 template <int WT>
-__device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, uint32_t g, const double* fit)
+__device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, uint32_t g, const double* fit,
+                                               const uint4& first)
 {
     uint32_t best = 0;
     double bf = 0.0;
     for (uint32_t d = 0; d < a.s; d += 4) {
-        const uint4 r = philox10(make_uint4(gid, g, TAG_SELECT, d >> 2), a.key0, a.key1);
+        const uint4 r = d == 0 ? first : philox10(make_uint4(gid, g, TAG_SELECT, d >> 2), a.key0, a.key1);
         uint32_t ids[4];
         double fs[4];
 #pragma unroll
@@ -1335,19 +1369,54 @@ __device__ __forceinline__ void init_row(const GaArgs& a, Row<WT>& row, uint32_t
 // each lane then builds only its own child (R8, R18).  32-child chunks are
 // dealt round-robin over every worker warp of the island (warp-major), so all
 // SMs get the same share.
+// Record snapshot of parity `par` of island i (f and, for narrow rows, bits)
+template <int WT>
+__device__ __forceinline__ BestRow<WT> load_snapshot(const GaArgs& a, uint32_t i, uint32_t par)
+{
+    BestRow<WT> s;
+    const uint32_t sp = par * a.I + i;
+    s.f = __ldcg(a.snap_f + sp);
+    s.idx = 0;
+#pragma unroll
+    for (int w = 0; w < WT; ++w) s.r.w[w] = (WT <= 8 && w < (int)a.ch.W) ? __ldcg(a.snap_bits + (size_t)sp * a.ch.W + w) : 0ull;
+    return s;
+}
+
+// Philox draws of one child for generation g (SELECT block 0, XOVER of its
+// pair, MUTATE), computed ahead of the generation barrier when possible.
+struct ChildDraws {
+    uint4 sel, xo, mu;
+};
+__device__ __forceinline__ ChildDraws child_draws(const GaArgs& a, uint32_t gid, uint32_t h, uint32_t g)
+{
+    ChildDraws d;
+    d.sel = philox10(make_uint4(gid, g, TAG_SELECT, 0), a.key0, a.key1);
+    d.xo = philox10(make_uint4(gid - h, g, TAG_XOVER, 0), a.key0, a.key1);
+    d.mu = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);
+    return d;
+}
+
+// One child per thread.  The two children of a pair (c0 = E + 2q, c1 = c0 + 1)
+// sit in adjacent lanes and swap their tournament winners with one shuffle;
+// each lane then builds only its own child (R8, R18).  32-child chunks are
+// dealt round-robin over every worker warp of the island (warp-major), so all
+// SMs get the same share.  Candidates for the next elite merge go to this
+// CTA's own region of the list (counted in shared memory, no global atomics).
 template <int WT>
 __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl,
                                                const uint64_t* popc, const double* fitc, uint64_t* popn,
                                                double* fitn, const uint32_t* sP, const uint32_t* sO,
-                                               const uint64_t* tau_ptr, uint32_t* ccnt, uint64_t* ckey,
-                                               uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx, uint32_t snap)
+                                               const uint64_t* tau_ptr, uint32_t* s_ccnt, uint64_t* ckey,
+                                               uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx,
+                                               const BestRow<WT>& snap, ChildDraws& pre, bool& have_pre)
 {
     const ChainDev& ch = a.ch;
     const uint32_t W = ch.W, N = a.N, E = a.E;
     const uint32_t nchild = N - E;
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const uint32_t chunks = (nchild + 31u) / 32u;
-    for (uint32_t cidx_ = warp * a.cpi + wl; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
+    const uint32_t first = warp * a.cpi + wl;
+    for (uint32_t cidx_ = first; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
         const uint32_t base = cidx_ * 32u;
         const uint32_t t = base + lane;
         const bool valid = t < nchild;
@@ -1356,7 +1425,10 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         const uint32_t gid = (a.island_base + i) * N + slot;
         const bool tr = kTrace && a.trace && threadIdx.x == 0 && blockIdx.x == a.I &&
                         g - a.g_begin < a.trace_gens && cidx_ == wl;
-        const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc) : 0u;     // a4
+        ChildDraws dr;
+        if (cidx_ == first && have_pre) dr = pre;
+        else dr = child_draws(a, gid, h, g);
+        const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc, dr.sel) : 0u;     // a4
         const uint32_t other = __shfl_xor_sync(0xFFFFFFFFu, mine, 1);
         if (tr) a.trace[(g - a.g_begin) * 16 + 8] = gtimer() + 0 * mine;
         if (!valid) continue;
@@ -1365,9 +1437,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         row_load(A, popc + (size_t)mine * W, W);
         row_load(B, popc + (size_t)other * W, W);
         if (tr) a.trace[(g - a.g_begin) * 16 + 9] = gtimer() + 0 * (A.w[0] ^ B.w[0]);
-        const uint4 rx = philox10(make_uint4(gid - h, g, TAG_XOVER, 0), a.key0, a.key1);   // a5
-        if ((uint64_t)rx.x < a.thr_c && ch.n >= 3) {
-            const uint32_t x = 1 + below(rx.y, ch.n - 2);
+        if ((uint64_t)dr.xo.x < a.thr_c && ch.n >= 3) {                                   // a5
+            const uint32_t x = 1 + below(dr.xo.y, ch.n - 2);
 #pragma unroll
             for (int w = 0; w < WT; ++w) {
                 const uint32_t lo = 64u * w;
@@ -1376,36 +1447,36 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
             }
         }
         if (tr) a.trace[(g - a.g_begin) * 16 + 13] = gtimer() + 0 * A.w[0];
-        const uint4 rm = philox10(make_uint4(gid, g, TAG_MUTATE, 0), a.key0, a.key1);     // a6
-        if ((uint64_t)rm.x < a.thr_m) row_xor_bit(A, below(rm.y, ch.n - 1));
+        if ((uint64_t)dr.mu.x < a.thr_m) row_xor_bit(A, below(dr.mu.y, ch.n - 1));      // a6
         repair(a, A, gid, g);                                                              // a7
         if (tr) a.trace[(g - a.g_begin) * 16 + 10] = gtimer() + 0 * A.w[0];
         const double f = eval_regs(ch, sP, sO, A, nullptr);                               // a2
         if (tr) a.trace[(g - a.g_begin) * 16 + 11] = gtimer() + 0 * (uint64_t)__double_as_longlong(f);
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
-        append_if(fkey(f) > __ldcg(tau_ptr), ccnt, ckey, cidx, fkey(f), slot);
+        append_if(fkey(f) > __ldcg(tau_ptr), s_ccnt, ckey, cidx, fkey(f), slot);
         if (tr) a.trace[(g - a.g_begin) * 16 + 14] = gtimer();
-        if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
         // a8 filter: only children that beat a snapshot of an earlier record of this
         // island (a lower bound of the current record) can change the record
-        const double snap_f = __ldcg(a.snap_f + snap);
-        bool improves = f > snap_f;
-        if (f == snap_f) {
-            if (WT > 16) {
-                improves = true;                      // wide rows: let the leader compare bits
+        bool improves = f > snap.f;
+        if (f == snap.f) {
+            if (WT > 8) {
+                improves = true;                      // wide rows: the leader compares bits
             } else {
                 bool decided = false;
 #pragma unroll
-                for (int w = WT - 1; w >= 0; --w) {
-                    if (w < (int)W && !decided) {
-                        const uint64_t sw = __ldcg(a.snap_bits + (size_t)snap * W + w);
-                        if (A.w[w] != sw) { improves = A.w[w] < sw; decided = true; }
-                    }
-                }
+                for (int w = WT - 1; w >= 0; --w)
+                    if (w < (int)W && !decided && A.w[w] != snap.r.w[w]) { improves = A.w[w] < snap.r.w[w]; decided = true; }
             }
         }
         append_if(improves, rcnt, nullptr, ridx, 0, slot);
+        if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
+    }
+    // draws of this thread's first child for generation g+1, ahead of the barrier
+    have_pre = first < chunks;
+    if (have_pre) {
+        const uint32_t t = first * 32u + lane;
+        pre = child_draws(a, (a.island_base + i) * N + E + t, t & 1u, g + 1);
     }
 }
 
@@ -1549,6 +1620,16 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
     // breed(g) appends generation g+1's to list (g+1)%3, leader(g) resets (g+2)%3.
     const bool first_full = __ldcg(&a.ctl->full) != 0;
     uint32_t mph = 0;
+    ChildDraws pre;
+    bool have_pre = false;
+    BestRow<WT> snap;
+    snap.f = -CUDART_INF;         // first phase of a launch: no filter (all children compared)
+    snap.idx = 0;
+#pragma unroll
+    for (int w = 0; w < WT; ++w) snap.r.w[w] = ~0ull;
+    if (worker) snap = load_snapshot<WT>(a, my_island, (a.g_begin + 1u) & 1u);   // REC(g_begin - 1), or INIT
+    if (threadIdx.x == 0) sm.misc[24] = 0;
+    __syncthreads();
     if (is_leader) {
         rec_load(a, blockIdx.x, sm);
         if (threadIdx.x == 0) {
@@ -1571,7 +1652,6 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
                 // the previous segment (and by the migrant import)
                 leader_general(a, blockIdx.x, g, sm);
                 if (threadIdx.x == 0) {
-                    a.cand_cnt[((g + 2u) % 3u) * I + blockIdx.x] = 0;
                     a.rc_cnt[((g + 2u) % 3u) * I + blockIdx.x] = 0;
                     if (blockIdx.x == 0) a.ctl->n_general = ++sm.misc[9];
                 }
@@ -1587,11 +1667,19 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             const uint32_t i = my_island;
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 4] = gtimer();
+            const size_t reg = ((size_t)i * cpi + my_local) * a.creg;    // this CTA's candidate region
             breed_children<WT>(a, i, g, my_local, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * Ns,
                                a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
-                               a.tau + tau_par * I + i, a.cand_cnt + Lb * I + i, a.cand_key[Lb] + (size_t)i * Ns,
-                               a.cand_idx[Lb] + (size_t)i * Ns, a.rc_cnt + Lb * I + i,
-                               a.rc_idx[Lb] + (size_t)i * Ns, nxt * I + i);
+                               a.tau + tau_par * I + i, sm.misc + 24, a.cand_key[Lb] + reg, a.cand_idx[Lb] + reg,
+                               a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre);
+            // snapshot for breed(g+1), read before the barrier: REC(g-1) (parity of g+1),
+            // stable during this phase and a lower bound of every later record
+            snap = load_snapshot<WT>(a, i, nxt);
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                a.cand_cnt[((size_t)Lb * I + i) * cpp + my_local] = sm.misc[24];    // publish, reset
+                sm.misc[24] = 0;
+            }
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
         }
