@@ -444,6 +444,7 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     TRY(dalloc(h, &a.mig_bits, (size_t)a.I_total * std::max<uint32_t>(a.K, 1) * h->W));
     TRY(dalloc(h, &a.mig_f, (size_t)a.I_total * std::max<uint32_t>(a.K, 1)));
     TRY(dalloc(h, &a.ctl, 1));
+    TRY(dalloc(h, &a.gbar, 4));
     TRY(dalloc(h, &h->d_stats, 8));
     TRY(dalloc(h, &h->d_statf, 1));
     TRY(dalloc(h, &h->d_bits1, h->W));
@@ -526,6 +527,10 @@ extern "C" int split_eval_batch_host(split_ga_t* h, const uint64_t* bits_host, u
 static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
 {
     GaArgs a = h->ga;
+    if (mode == MODE_RUN) {
+        cudaError_t me = cudaMemsetAsync(a.gbar, 0, 16, h->stream);
+        if (me != cudaSuccess) return fail(SPLIT_E_CUDA, "barrier reset: %s", cudaGetErrorString(me));
+    }
     a.mode = mode;
     a.trace = (mode == MODE_RUN) ? h->d_trace : nullptr;
     a.trace_gens = h->trace_gens;

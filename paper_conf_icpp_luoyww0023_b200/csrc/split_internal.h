@@ -79,6 +79,7 @@ struct GaArgs {
     double* snap_f;                    // [2][I] record snapshots (parity g&1), read by breed(g+1)
     uint64_t* snap_bits;               // [2][I][W]
     Ctl* ctl;
+    unsigned int* gbar;                // generation barrier counter (RUN launches)
     unsigned long long* trace;         // optional phase timestamps (SPLIT_TRACE), [trace_gens][8]
     uint32_t trace_gens;
 };

@@ -133,6 +133,25 @@ __device__ __forceinline__ void trace_mark(const GaArgs& a, uint32_t g, uint32_t
     if (gi < a.trace_gens) a.trace[gi * 16 + slot] = gtimer();
 }
 
+// Split grid barrier for the generation loop (all CTAs are co-resident: the
+// kernel is a cooperative launch).  arrive: CTA-ordered writes are released at
+// gpu scope by one red.release; wait: one thread polls with ld.acquire.
+__device__ __forceinline__ void gbar_arrive(unsigned int* ctr)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
+}
+__device__ __forceinline__ void gbar_wait(const unsigned int* ctr, unsigned int target)
+{
+    if (threadIdx.x == 0) {
+        unsigned int v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+        } while ((int)(v - target) < 0);
+    }
+    __syncthreads();
+}
+
 // asynchronous global->shared copies (LDGSTS), no register staging
 __device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc)
 {
@@ -1472,11 +1491,18 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         append_if(improves, rcnt, nullptr, ridx, 0, slot);
         if (tr) a.trace[(g - a.g_begin) * 16 + 12] = gtimer();
     }
-    // draws of this thread's first child for generation g+1, ahead of the barrier
+}
+
+// draws of this thread's first child for generation g+1 (overlaps the barrier)
+__device__ __forceinline__ void precompute_draws(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl,
+                                                 ChildDraws& pre, bool& have_pre)
+{
+    const uint32_t nchild = a.N - a.E, chunks = (nchild + 31u) / 32u;
+    const uint32_t first = (threadIdx.x >> 5) * a.cpi + wl;
     have_pre = first < chunks;
     if (have_pre) {
-        const uint32_t t = first * 32u + lane;
-        pre = child_draws(a, (a.island_base + i) * N + E + t, t & 1u, g + 1);
+        const uint32_t t = first * 32u + (threadIdx.x & 31u);
+        pre = child_draws(a, (a.island_base + i) * a.N + a.E + t, t & 1u, g + 1);
     }
 }
 
@@ -1622,6 +1648,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
     uint32_t mph = 0;
     ChildDraws pre;
     bool have_pre = false;
+    unsigned int bar_target = 0;      // generation barrier counter (zeroed by the host per launch)
     BestRow<WT> snap;
     snap.f = -CUDART_INF;         // first phase of a launch: no filter (all children compared)
     snap.idx = 0;
@@ -1683,7 +1710,10 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
         }
-        grid.sync();
+        gbar_arrive(a.gbar);
+        if (worker) precompute_draws(a, my_island, g, my_local, pre, have_pre);
+        bar_target += gridDim.x;
+        gbar_wait(a.gbar, bar_target);
         if (kTrace && threadIdx.x == 0 && a.trace && g - a.g_begin < a.trace_gens) {
             if (blockIdx.x == 0) a.trace[(g - a.g_begin) * 16 + 6] = gtimer();
             if (blockIdx.x == I) a.trace[(g - a.g_begin) * 16 + 7] = gtimer();
