@@ -118,13 +118,6 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
-def _dist_env():
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    return world, rank, local
-
-
 def ga_bytes_per_generation(N: int, E: int, W: int, s: int) -> int:
     """Algorithmic HBM bytes of one generation: per child one parent row
     read (pairs read two rows for two children), one child row and one f64 written, s
@@ -151,7 +144,7 @@ def cpu_baseline_oracle(generations: int) -> dict:
 
 
 def run_reference(args):
-    world, rank, _ = _dist_env()
+    rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
     import oracle
@@ -198,23 +191,23 @@ def main():
 
     import torch
     import torch.distributed as dist
+    from paper_conf_icpp_luoyww0023_b200 import dist as D
     from paper_conf_icpp_luoyww0023_b200 import split as S
     from paper_conf_icpp_luoyww0023_b200 import workloads as wl
 
-    world, rank, local = _dist_env()
+    rank, world, local = D.env_rank_world()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     comm = None
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-        uid = [S.split_comm_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        comm = S.split_comm_init(uid[0], rank, world, local)
+        uid = D.broadcast_bytes(S.split_comm_unique_id() if rank == 0 else None)
+        comm = S.split_comm_init(uid, rank, world, local)
     stream = torch.cuda.current_stream()
     lat, ovh = wl.chain(C2["chain"])
     G = args.generations
     gkw = {k: C2[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max")}
-    isl = dict(island_id=rank, n_islands=world, islands_per_device=1,
+    isl = dict(**D.island_layout(rank, world, 1),
                migration_interval=MIGRATION_INTERVAL if world > 1 else 0, n_migrants=N_MIGRANTS if world > 1 else 0)
     h = S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl)
     W = h.W
@@ -255,13 +248,8 @@ def main():
     for i in range(args.steps):
         step_ms.append(ev0[i].elapsed_time(ev1[i]))
     t_ms = sum(step_ms)
-    t = torch.tensor([t_ms, wall * 1000.0], dtype=torch.float64, device=dev)
-    tot = torch.tensor([float(evals), float(gens)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
-    t_max_ms, wall_max_ms = float(t[0]), float(t[1])
-    evals_all = float(tot[0])
+    t_max_ms, evals_all, _ = D.reduce_max_sum(t_ms, float(evals), float(gens), device=dev)
+    wall_max_ms, _, _ = D.reduce_max_sum(wall * 1000.0, 0.0, device=dev)
     value = evals_all / (t_max_ms / 1000.0)
     gens_per_s = (gens / (t_max_ms / 1000.0))           # generations of the GA (island-parallel)
 
@@ -332,15 +320,11 @@ def main():
                 e_evals += he.run(G, 5000 + i)["evaluations"]
         torch.cuda.synchronize()
         barrier()
-        et = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
-        ee = torch.tensor([float(e_evals)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(et, op=dist.ReduceOp.MAX)
-            dist.all_reduce(ee, op=dist.ReduceOp.SUM)
+        et_s, ee_all, _ = D.reduce_max_sum(time.perf_counter() - t0, float(e_evals), device=dev)
         n = len(lat)
         h2d = 4 * (((n + 1 + 3) & ~3) + ((n - 1 + 3) & ~3)) + 8   # staged chain words + best bits
         d2h = 48 + world * (W + 2) * 8 + 5 * 8 + 8                # control block, island records, best stats
-        out["e2e"] = {"value": float(ee[0]) / float(et[0]), "unit": UNIT, "h2d_bytes_per_step": h2d,
+        out["e2e"] = {"value": ee_all / et_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
                       "d2h_bytes_per_step": d2h, "steps": e2e_steps,
                       "note": "split_ga_create(host latencies) + split_ga_run + best to host + destroy, wall clock"}
 

@@ -141,3 +141,26 @@ def test_c2_full_run_invariants(S):
     s = oracle.fitness(lat, ovh, r["bits"], 2, 32)
     assert s["fitness"] == r["fitness"] and s["var_num"] == r["var_num"] and s["k"] == r["k"]
     assert r["expected_wait_ns"] == pytest.approx(s["s2"] / (2 * s["s1"]))
+
+
+def test_islands_through_nccl_communicator(S):
+    """The island exchange through a (1-rank) NCCL communicator: same trajectory
+    as the oracle's serial islands (the all-gathers run in NCCL)."""
+    uid = S.split_comm_unique_id()
+    comm = S.split_comm_init(uid, 0, 1, 0)
+    try:
+        lat, ovh = wl.chain("resnet50_175")
+        kw = dict(pop_size=256, n_elite=8, k_min=2, k_max=16, n_islands=4, islands_per_device=4,
+                  migration_interval=3, n_migrants=8)
+        h = S.SplitGA(lat, ovh, comm=comm, **kw)
+        r = h.run(10, 5)
+        pops = [h.population(i) for i in range(4)]
+        h.close()
+    finally:
+        S.split_comm_destroy(comm)
+    o = oracle.ga_run(lat, ovh, 10, 5, want_population=True,
+                      **{k: v for k, v in kw.items() if k in ORACLE_KEYS})
+    assert r["fitness"] == o["fitness"] and np.array_equal(r["bits"], o["bits"])
+    assert r["generation_found"] == o["generation_found"]
+    for i in range(4):
+        assert np.array_equal(pops[i][0], o["population"][i])
