@@ -465,25 +465,25 @@ __global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_w_kernel(ChainDev 
             const uint32_t k = cuts + 1;
             double f = -CUDART_INF;
             if (k >= ch.k_min && k <= ch.k_max) {
-                uint32_t startP = 0, prev_o = 0, OV = 0, v = 0, q = 0;
+                // walk the cuts from the last one down (one FLO per cut): the block
+                // after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+                uint32_t endP = ch.T, OV = 0, v = 0, q = 0;
                 uint64_t S2 = 0;
                 for (uint32_t j = 0; j < cuts; ++j) {
                     if (v == 0u) {
-                        q = __ffs(occ) - 1;
-                        occ &= occ - 1;
+                        q = 31u - __clz(occ);
+                        occ ^= 1u << q;
                         v = my[q];
                     }
-                    const uint32_t p = 32u * q + (uint32_t)(__ffs(v) - 1);
-                    v &= v - 1;
-                    const uint2 e = spo[p];
-                    const uint32_t tj = e.x - startP + prev_o;
+                    const uint32_t bt = 31u - __clz(v);
+                    v ^= 1u << bt;
+                    const uint2 e = spo[32u * q + bt];
+                    const uint32_t tj = endP - e.x + e.y;
                     S2 += (uint64_t)tj * tj;
                     OV += e.y;
-                    startP = e.x;
-                    prev_o = e.y;
+                    endP = e.x;
                 }
-                const uint32_t tl = ch.T - startP + prev_o;
-                S2 += (uint64_t)tl * tl;
+                S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
                 const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
                 const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
                 f = eq2(k, V, OV, ch.T);
