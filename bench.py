@@ -71,26 +71,37 @@ def _profile_traffic(name: str):
 
 
 class ClockSampler:
-    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+    """nvidia-smi clock / throttle-reason sampler; summary() keeps the samples whose
+    timestamps fall inside the timed region (mark_start / mark_end)."""
+    FIELDS = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
 
     def __init__(self, device: int):
         self.device = device
         self.proc = None
+        self.t0 = self.t1 = None
 
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(
-                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100",
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "50",
                  "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.5)                       # let the sampler start before the timed region
         except Exception:
             self.proc = None
         return self
 
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_end(self):
+        self.t1 = time.time()
+
     def __exit__(self, *exc):
         self.lines = []
         if self.proc:
+            time.sleep(0.1)
             self.proc.terminate()
             try:
                 out, _ = self.proc.communicate(timeout=5)
@@ -100,22 +111,27 @@ class ClockSampler:
             self.lines = [ln for ln in out.splitlines() if ln.strip()]
 
     def summary(self) -> dict:
-        sm, mx, reasons = [], None, set()
+        import datetime
+        sm, mx, reasons, inside = [], None, set(), 0
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in getattr(self, "lines", []):
             parts = [x.strip() for x in ln.split(",")]
-            if len(parts) < 8:
+            if len(parts) < 9:
                 continue
             try:
-                sm.append(float(parts[1]))
-                mx = float(parts[2])
+                ts = datetime.datetime.strptime(parts[0], "%Y/%m/%d %H:%M:%S.%f").timestamp()
+                clk, mx = float(parts[2]), float(parts[3])
             except ValueError:
                 continue
-            for nm, v in zip(names, parts[4:8]):
+            if self.t0 is not None and not (self.t0 - 0.05 <= ts <= (self.t1 or ts) + 0.05):
+                continue
+            inside += 1
+            sm.append(clk)
+            for nm, v in zip(names, parts[5:9]):
                 if v.lower().startswith("active"):
                     reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+                "samples": inside}
 
 
 def ga_bytes_per_generation(N: int, E: int, W: int, s: int) -> int:
@@ -176,7 +192,7 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--generations", type=int, default=C2["generations"])
@@ -228,6 +244,7 @@ def main():
     with ClockSampler(local) as clk:
         barrier()
         torch.cuda.synchronize()
+        clk.mark_start()
         wall0 = time.perf_counter()
         for i in range(args.steps):
             flush.fill_(i & 0xFF)                    # L2 flush between timed steps (not timed)
@@ -245,6 +262,7 @@ def main():
         torch.cuda.synchronize()
         barrier()
         wall = time.perf_counter() - wall0
+        clk.mark_end()
     for i in range(args.steps):
         step_ms.append(ev0[i].elapsed_time(ev1[i]))
     t_ms = sum(step_ms)
@@ -261,7 +279,7 @@ def main():
     roofline = {"bound": "hbm", "kernel": "ga_kernel (RUN segment: all generations of a step)",
                 "achieved": achieved_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved_gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
-                "traffic": _profile_traffic("ga_kernel_per_generation"),
+                "traffic": _profile_traffic("ga_kernel_per_launch"),
                 "algorithmic_bytes_per_generation": gen_bytes,
                 "launch_ms_avg": loop_avg_ms, "share_of_step": loop_avg_ms / (t_max_ms / args.steps)}
 
