@@ -1,498 +1,8 @@
-// split_kernels.cu — sm_100a kernels of the GA split search (SPLIT, ICPP'23 §3.3).
-//
-// K1  eval_batch_kernel   a2: bitset -> (k, S1, S2, V, OV) exact integers -> Eq. 2 in FP64
-//                          (PAPER.md P@21101-21296).  Chain prefix/overheads staged into
-//                          shared memory with one TMA bulk copy (cp.async.bulk + mbarrier);
-//                          bitset tiles loaded with coalesced 128-bit loads per warp.
-// K2+ ga_kernel            cooperative persistent kernel, one launch per GA segment:
-//                          a1 init (Philox + Floyd), a3 elite top-E (radix select over the
-//                          96-bit (fitness key, ~index) order, or a single-CTA merge of the
-//                          previous elites with the few children that beat the worst elite),
-//                          a4-a7 breed (tournament, one-point crossover, one-bit mutation,
-//                          rank-select repair) fused with a2 eval of the children, a8 best
-//                          record + stall, a9 migration export/import.
-// Everything is integer / FP64 scalar work: no tensor cores (north_star).
-// Determinism: every random draw is Philox4x32-10 keyed on (seed) with counter
-// (global individual, generation, tag, draw/4) (R9), and every
-// reduction breaks ties by index or bitset, so results match the CPU oracle
-// bit for bit.
-#include <cooperative_groups.h>
-#include <cuda_runtime.h>
-#include <math_constants.h>
-#include <stdint.h>
-
-#include "split_internal.h"
-
-namespace cg = cooperative_groups;
+// split_ga.cu — the cooperative persistent GA kernel (a1, a3-a9) of SPLIT's
+// split search (ICPP'23 §3.3) and its launchers; see DESIGN.md §5.
+#include "split_device.cuh"
 
 namespace splitga {
-
-constexpr uint32_t NONE = 0xFFFFFFFFu;
-#ifdef SPLIT_TRACE_BUILD
-constexpr bool kTrace = true;     // phase timestamps (tools: SPLIT_TRACE=<csv>)
-#else
-constexpr bool kTrace = false;
-#endif
-
-// ------------------------------------------------------------------------
-// Philox4x32-10 (Salmon et al., SC'11), multipliers/Weyl constants of the
-// Random123 reference.  Device-side implementation, independent of oracle/.
-// ------------------------------------------------------------------------
-__device__ __forceinline__ uint4 philox10(uint4 c, uint32_t k0, uint32_t k1)
-{
-#pragma unroll
-    for (int r = 0; r < 10; ++r) {
-        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = __umulhi(0xD2511F53u, c.x);
-        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = __umulhi(0xCD9E8D57u, c.z);
-        c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
-        k0 += 0x9E3779B9u;
-        k1 += 0xBB67AE85u;
-    }
-    return c;
-}
-
-__device__ __forceinline__ uint32_t lane_of(const uint4& v, uint32_t l)
-{
-    return l == 0 ? v.x : (l == 1 ? v.y : (l == 2 ? v.z : v.w));
-}
-
-// sequential draws d = 0, 1, ... of one (id, gen, tag) stream
-struct Draws {
-    uint32_t id, gen, tag, d, k0, k1;
-    uint4 blk;
-    __device__ __forceinline__ Draws(uint32_t id_, uint32_t gen_, uint32_t tag_, uint32_t k0_, uint32_t k1_)
-        : id(id_), gen(gen_), tag(tag_), d(0), k0(k0_), k1(k1_) {}
-    __device__ __forceinline__ uint32_t next()
-    {
-        if ((d & 3u) == 0) blk = philox10(make_uint4(id, gen, tag, d >> 2), k0, k1);
-        return lane_of(blk, (d++) & 3u);
-    }
-};
-
-// uniform integer in [0, m): floor(u * m / 2^32)
-__device__ __forceinline__ uint32_t below(uint32_t u, uint32_t m) { return __umulhi(u, m); }
-
-// ------------------------------------------------------------------------
-// dexp: exp by the fixed operation sequence of DESIGN.md R5'' (Cody-Waite
-// reduction, degree-13 Taylor polynomial in Horner form, RN(1/i!)).
-// ------------------------------------------------------------------------
-__device__ __forceinline__ double dexp_dev(double z)
-{
-    if (z > 710.0) return CUDART_INF;
-    if (z < -700.0) return 0.0;
-    // j = rint(z / ln 2), ties to even: adding 1.5*2^52 rounds to an integer (RN)
-    const double t = __dadd_rn(__dmul_rn(z, 0x1.71547652b82fep+0), 0x1.8p52);
-    const double j = __dsub_rn(t, 0x1.8p52);
-    const int ji = (int)(uint32_t)__double_as_longlong(t);     // low word of t holds j
-    double r = __fma_rn(-j, 0x1.62e42fefa39efp-1, z);
-    r = __fma_rn(-j, 0x1.abc9e3b39803fp-56, r);
-    double p = 0x1.6124613a86d09p-33;           // 1/13!
-    p = __fma_rn(p, r, 0x1.1eed8eff8d898p-29);  // 1/12!
-    p = __fma_rn(p, r, 0x1.ae64567f544e4p-26);  // 1/11!
-    p = __fma_rn(p, r, 0x1.27e4fb7789f5cp-22);  // 1/10!
-    p = __fma_rn(p, r, 0x1.71de3a556c734p-19);  // 1/9!
-    p = __fma_rn(p, r, 0x1.a01a01a01a01ap-16);  // 1/8!
-    p = __fma_rn(p, r, 0x1.a01a01a01a01ap-13);  // 1/7!
-    p = __fma_rn(p, r, 0x1.6c16c16c16c17p-10);  // 1/6!
-    p = __fma_rn(p, r, 0x1.1111111111111p-7);   // 1/5!
-    p = __fma_rn(p, r, 0x1.5555555555555p-5);   // 1/4!
-    p = __fma_rn(p, r, 0x1.5555555555555p-3);   // 1/3!
-    p = __fma_rn(p, r, 0.5);
-    p = __fma_rn(p, r, 1.0);
-    p = __fma_rn(p, r, 1.0);
-    // ldexp(p, j) for j in [-2, 1024]: exact scaling by powers of two (p in [0.7, 1.5])
-    const int j1 = ji > 1023 ? 1023 : ji;
-    const double s1 = __longlong_as_double((long long)(j1 + 1023) << 52);
-    const double s2 = __longlong_as_double((long long)(ji - j1 + 1023) << 52);
-    return __dmul_rn(__dmul_rn(p, s1), s2);
-}
-
-// Eq. 2 from the exact integer statistics (R5'):
-//   x = sigma/T = sqrt(V)/(k T),  y = overhead/m = (OV/T)/k,  f = -(e^(x-1) + e^(y-1))
-__device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, uint32_t T)
-{
-    const double Td = __uint2double_rn(T);
-    const double kd = __uint2double_rn(k);
-    const double x = __ddiv_rn(__dsqrt_rn(__ll2double_rn(V)), __dmul_rn(kd, Td));
-    const double y = __ddiv_rn(__ddiv_rn(__ull2double_rn(OV), Td), kd);
-    return -__dadd_rn(dexp_dev(__dsub_rn(x, 1.0)), dexp_dev(__dsub_rn(y, 1.0)));
-}
-
-__device__ __forceinline__ unsigned long long gtimer()
-{
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    return t;
-}
-// phase timestamps (SPLIT_TRACE): leader CTA 0 slots 0-3, last worker CTA 4-5,
-// after the generation barrier 6 (CTA 0) and 7 (last CTA)
-__device__ __forceinline__ void trace_mark(const GaArgs& a, uint32_t g, uint32_t slot)
-{
-    if (!kTrace || !a.trace || threadIdx.x != 0 || blockIdx.x != 0) return;
-    const uint32_t gi = g - a.g_begin;
-    if (gi < a.trace_gens) a.trace[gi * 16 + slot] = gtimer();
-}
-
-// Split grid barrier for the generation loop (all CTAs are co-resident: the
-// kernel is a cooperative launch).  arrive: CTA-ordered writes are released at
-// gpu scope by one red.release; wait: one thread polls with ld.acquire.
-__device__ __forceinline__ void gbar_arrive(unsigned int* ctr)
-{
-    __syncthreads();
-    if (threadIdx.x == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
-}
-__device__ __forceinline__ void gbar_wait(const unsigned int* ctr, unsigned int target)
-{
-    if (threadIdx.x == 0) {
-        unsigned int v;
-        do {
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-        } while ((int)(v - target) < 0);
-    }
-    __syncthreads();
-}
-
-// asynchronous global->shared copies (LDGSTS), no register staging
-__device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc)
-{
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"((uint32_t)__cvta_generic_to_shared(smem_dst)),
-                 "l"(gsrc)
-                 : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc)
-{
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(smem_dst)),
-                 "l"(gsrc)
-                 : "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
-// order-preserving u64 key of a fitness (larger f -> larger key)
-__device__ __forceinline__ uint64_t fkey(double f)
-{
-    const uint64_t u = (uint64_t)__double_as_longlong(f);
-    return (u >> 63) ? ~u : (u | 0x8000000000000000ull);
-}
-__device__ __forceinline__ double unkey(uint64_t k)
-{
-    const uint64_t u = (k >> 63) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
-    return __longlong_as_double((long long)u);
-}
-
-// ------------------------------------------------------------------------
-// Chain staging: one TMA bulk copy of P|ovh into shared memory.
-// ------------------------------------------------------------------------
-__device__ __forceinline__ void stage_chain(uint32_t* s_chain, const ChainDev& ch, uint64_t* mbar)
-{
-    const uint32_t bytes = (ch.p_words + ch.o_words) * 4u;   // multiple of 16
-    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
-    if (threadIdx.x == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(s_chain);
-        const uint32_t chunk = 32768u;
-        for (uint32_t off = 0; off < bytes; off += chunk) {
-            const uint32_t b = (bytes - off < chunk) ? (bytes - off) : chunk;
-            asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst + off),
-                "l"((const char*)ch.words + off), "r"(b), "r"(bar)
-                : "memory");
-        }
-    }
-    uint32_t ok = 0;
-    while (!ok) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
-            : "=r"(ok)
-            : "r"(bar)
-            : "memory");
-    }
-}
-
-// ------------------------------------------------------------------------
-// mbarrier + TMA bulk copies (cp.async.bulk) for the leader's loads
-// ------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count)
-{
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count));
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* mbar, uint32_t bytes)
-{
-    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* mbar, uint32_t bytes)
-{
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t parity)
-{
-    uint32_t ok = 0;
-    while (!ok) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-            : "=r"(ok)
-            : "r"(smem_u32(mbar)), "r"(parity)
-            : "memory");
-    }
-}
-// bytes: multiple of 16; src/dst 16-byte aligned
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* mbar)
-{
-    const uint32_t d = smem_u32(dst), b = smem_u32(mbar);
-    for (uint32_t off = 0; off < bytes; off += 32768u) {
-        const uint32_t n = (bytes - off < 32768u) ? (bytes - off) : 32768u;
-        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d + off),
-                     "l"((const char*)src + off), "r"(n), "r"(b)
-                     : "memory");
-    }
-}
-// Stage `bytes` (multiple of 16) of global memory into shared memory with TMA
-// bulk copies completing on one mbarrier; all threads return after arrival.
-__device__ __forceinline__ void stage_bulk(void* s_dst, const void* src, uint32_t bytes, uint64_t* mbar)
-{
-    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
-    if (threadIdx.x == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(s_dst);
-        for (uint32_t off = 0; off < bytes; off += 32768u) {
-            const uint32_t b = (bytes - off < 32768u) ? (bytes - off) : 32768u;
-            asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst + off),
-                "l"((const char*)src + off), "r"(b), "r"(bar)
-                : "memory");
-        }
-    }
-    uint32_t ok = 0;
-    while (!ok) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
-            : "=r"(ok)
-            : "r"(bar)
-            : "memory");
-    }
-}
-
-// Walk the cuts of one candidate: words come from `get(w)` in ascending order.
-// Block j ends at cut c_j; t_j = P[c_j+1] - P[c_{j-1}+1] + ovh[c_{j-1}] (R3).
-struct Stats {
-    uint32_t k;
-    int64_t V;
-    uint64_t S1, S2, OV;
-};
-
-template <class Get>
-__device__ __forceinline__ double eval_walk(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO, Get get,
-                                            Stats* st)
-{
-    uint32_t cuts = 0;
-    for (uint32_t w = 0; w < ch.W; ++w) {
-        uint64_t v = get(w);
-        if (w == ch.W - 1) v &= ch.last_mask;
-        cuts += __popcll(v);
-    }
-    const uint32_t k = cuts + 1;
-    if (k < ch.k_min || k > ch.k_max) {
-        if (st) st->k = k;
-        return -CUDART_INF;
-    }
-    uint32_t startP = 0, prev_o = 0;
-    uint64_t S1 = 0, S2 = 0, OV = 0;
-    for (uint32_t w = 0; w < ch.W; ++w) {
-        uint64_t v = get(w);
-        if (w == ch.W - 1) v &= ch.last_mask;
-        while (v) {
-            const uint32_t p = w * 64u + (uint32_t)(__ffsll((long long)v) - 1);
-            v &= v - 1;
-            const uint32_t Pp = sP[p + 1];
-            const uint32_t t = Pp - startP + prev_o;
-            S1 += t;
-            S2 += (uint64_t)t * t;
-            prev_o = sO[p];
-            OV += prev_o;
-            startP = Pp;
-        }
-    }
-    const uint32_t t = ch.T - startP + prev_o;
-    S1 += t;
-    S2 += (uint64_t)t * t;
-    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);   // exact: V < 2^63 by the a0 guard
-    if (st) { st->k = k; st->V = V; st->S1 = S1; st->S2 = S2; st->OV = OV; }
-    return eq2(k, V, OV, ch.T);
-}
-
-// ------------------------------------------------------------------------
-// K1: split_eval_batch.  Each warp stages 32 rows (coalesced 128-bit loads)
-// into a padded shared tile (odd pitch: conflict-free row reads), then every
-// lane walks its own candidate.
-// ------------------------------------------------------------------------
-constexpr int kEvalWarps = 8;
-
-__global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
-                                                                     uint64_t n_cand, double* __restrict__ out)
-{
-    extern __shared__ __align__(16) uint8_t smem[];
-    uint32_t* s_chain = (uint32_t*)smem;
-    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
-    uint64_t* s_tiles = mbar + 2;
-    const uint32_t W = ch.W;
-    const uint32_t pitch = W | 1u;
-    stage_chain(s_chain, ch, mbar);
-    const uint32_t* sP = s_chain;
-    const uint32_t* sO = s_chain + ch.p_words;
-
-    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    uint64_t* tile = s_tiles + (size_t)warp * 32u * pitch;
-    const uint64_t n_tiles = (n_cand + 31) / 32;
-    const uint64_t gw = (uint64_t)blockIdx.x * kEvalWarps + warp;
-    const uint64_t nw = (uint64_t)gridDim.x * kEvalWarps;
-    for (uint64_t t = gw; t < n_tiles; t += nw) {
-        const uint64_t row0 = t * 32;
-        const uint32_t rows = (uint32_t)((n_cand - row0) < 32 ? (n_cand - row0) : 32);
-        const uint64_t* src = bits + row0 * W;
-        const uint32_t nwords = rows * W;
-        if (rows == 32) {
-            const uint4* src4 = (const uint4*)src;        // 256*W bytes, 16-byte aligned
-            const uint32_t n4 = 16u * W;
-#pragma unroll 4
-            for (uint32_t j = lane; j < n4; j += 32) {
-                const uint4 v = __ldcs(src4 + j);
-                const uint32_t w0 = 2 * j, w1 = 2 * j + 1;
-                tile[(w0 / W) * pitch + (w0 % W)] = ((uint64_t)v.y << 32) | v.x;
-                tile[(w1 / W) * pitch + (w1 % W)] = ((uint64_t)v.w << 32) | v.z;
-            }
-        } else {
-            for (uint32_t j = lane; j < nwords; j += 32) tile[(j / W) * pitch + (j % W)] = __ldcs(src + j);
-        }
-        __syncwarp();
-        if (lane < rows) {
-            const uint64_t* my = tile + lane * pitch;
-            const double f = eval_walk(ch, sP, sO, [&](uint32_t w) { return my[w]; }, nullptr);
-            __stcs(out + row0 + lane, f);
-        }
-        __syncwarp();
-    }
-}
-
-// K1 for W <= 16 (n_ops <= 1025): W is a compile-time constant, rows are
-// handled as 2W 32-bit half-words and each lane keeps a bitmask of its
-// non-empty half-words, so the walk takes exactly one iteration per cut
-// (no per-word loop whose trip count diverges across the warp).
-// K1 for W <= 16.  Each warp streams 32-row tiles (32*W u64, contiguous) into
-// a double-buffered shared tile with TMA bulk copies (cp.async.bulk + one
-// mbarrier per buffer), so no instructions are spent staging.  Lane l owns row
-// l: a skewed pass (lane l reads half-word (q+l)%H at step q: conflict-free)
-// counts cuts and builds a bitmask of non-empty half-words, then the walk takes
-// exactly one iteration per cut.
-template <int W>
-__global__ void __launch_bounds__(kEvalWarps * 32) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
-                                                                       uint64_t n_cand, double* __restrict__ out)
-{
-    constexpr uint32_t H = 2 * W;          // 32-bit halves per row
-    constexpr uint32_t TILE = 32 * H;      // u32 per tile
-    extern __shared__ __align__(16) uint8_t smem[];
-    // staged chain: po[p] = {P[p+1], ovh[p]} for cut positions p in [0, n-2]
-    const uint2* spo = (const uint2*)smem;
-    uint64_t* mbar = (uint64_t*)(smem + ch.po_bytes);            // [0] chain, [1 + 2*warp + b] tiles
-    uint32_t* s_tiles = (uint32_t*)(mbar + 2 * kEvalWarps + 2);  // 16-byte aligned
-    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    uint64_t* wbar = mbar + 2 + 2 * warp;
-    if (lane == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(wbar)));
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(wbar + 1)));
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    stage_bulk(smem, ch.po, ch.po_bytes, mbar);                   // includes a __syncthreads
-    uint32_t* tiles = s_tiles + warp * 2u * TILE;
-    const uint32_t npos = ch.n - 1, qfull = npos >> 5;
-    const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
-    const uint64_t n_full = n_cand / 32;                           // full tiles go through TMA
-    const uint64_t n_tiles = (n_cand + 31) / 32;
-    const uint64_t nw = (uint64_t)gridDim.x * kEvalWarps;
-    uint64_t t = (uint64_t)blockIdx.x * kEvalWarps + warp;
-    auto issue = [&](uint64_t tt, uint32_t b) {
-        if (lane == 0 && tt < n_full) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            mbar_arrive_expect_tx(wbar + b, TILE * 4u);
-            bulk_g2s(tiles + b * TILE, bits + tt * 32 * W, TILE * 4u, wbar + b);
-        }
-    };
-    issue(t, 0);
-    uint32_t ph = 0;                       // bit b: parity of buffer b's next phase
-    for (uint32_t b = 0; t < n_tiles; t += nw, b ^= 1u) {
-        issue(t + nw, b ^ 1u);
-        uint32_t* tile = tiles + b * TILE;
-        const uint64_t row0 = t * 32;
-        const uint32_t rows = (uint32_t)((n_cand - row0) < 32 ? (n_cand - row0) : 32);
-        if (t < n_full) {
-            mbar_wait(wbar + b, (ph >> b) & 1u);
-            ph ^= 1u << b;
-        } else {
-            const uint32_t* src = (const uint32_t*)(bits + row0 * W);
-            for (uint32_t e = lane; e < rows * H; e += 32) tile[e] = __ldcs(src + e);
-            __syncwarp();
-        }
-        if (lane < rows) {
-            uint32_t* my = tile + lane * H;
-            uint32_t cuts = 0, occr = 0;
-#pragma unroll
-            for (uint32_t q = 0; q < H; ++q) {
-                const uint32_t v = my[(q + lane) % H];
-                cuts += __popc(v);
-                occr |= (v != 0u ? 1u : 0u) << q;
-            }
-            // bit q of occr is half (q + lane) % H: rotate into place
-            uint32_t occ = (H == 32) ? __funnelshift_l(occr, occr, lane)
-                                     : (((occr << (lane % H)) | (occr >> ((H - lane % H) % H))) & (H == 32 ? ~0u : ((1u << H) - 1u)));
-            // padding (positions >= n-1): only halves >= qfull, usually one
-            for (uint32_t q = qfull; q < H; ++q) {
-                const uint32_t v = my[q];
-                const uint32_t keep = (q == qfull) ? (v & lastm) : 0u;
-                cuts -= __popc(v ^ keep);
-                my[q] = keep;
-                if (!keep) occ &= ~(1u << q);
-            }
-            const uint32_t k = cuts + 1;
-            double f = -CUDART_INF;
-            if (k >= ch.k_min && k <= ch.k_max) {
-                // walk the cuts from the last one down (one FLO per cut): the block
-                // after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
-                uint32_t endP = ch.T, OV = 0, v = 0, q = 0;
-                uint64_t S2 = 0;
-                for (uint32_t j = 0; j < cuts; ++j) {
-                    if (v == 0u) {
-                        q = 31u - __clz(occ);
-                        occ ^= 1u << q;
-                        v = my[q];
-                    }
-                    const uint32_t bt = 31u - __clz(v);
-                    v ^= 1u << bt;
-                    const uint2 e = spo[32u * q + bt];
-                    const uint32_t tj = endP - e.x + e.y;
-                    S2 += (uint64_t)tj * tj;
-                    OV += e.y;
-                    endP = e.x;
-                }
-                S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
-                const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
-                const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
-                f = eq2(k, V, OV, ch.T);
-            }
-            __stcs(out + row0 + lane, f);
-        }
-        __syncwarp();
-    }
-}
 
 // ------------------------------------------------------------------------
 // GA kernel helpers
@@ -1739,87 +1249,8 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
 }
 
 // ------------------------------------------------------------------------
-// Small kernels
-// ------------------------------------------------------------------------
-__global__ void eval_stats_kernel(ChainDev ch, const uint64_t* bits, int64_t* st_out, double* f_out)
-{
-    extern __shared__ __align__(16) uint8_t smem[];
-    uint32_t* s_chain = (uint32_t*)smem;
-    uint64_t* mbar = (uint64_t*)(smem + (ch.p_words + ch.o_words) * 4u);
-    stage_chain(s_chain, ch, mbar);
-    if (threadIdx.x == 0) {
-        Stats st{};
-        const double f = eval_walk(ch, s_chain, s_chain + ch.p_words, [&](uint32_t w) { return bits[w]; }, &st);
-        st_out[0] = st.k; st_out[1] = st.V; st_out[2] = (int64_t)st.S1; st_out[3] = (int64_t)st.S2; st_out[4] = (int64_t)st.OV;
-        *f_out = f;
-    }
-}
-
-__global__ void selftest_philox_kernel(const uint32_t* in, uint32_t n, uint32_t* out)
-{
-    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= n) return;
-    const uint32_t* v = in + 6 * t;
-    const uint4 r = philox10(make_uint4(v[0], v[1], v[2], v[3]), v[4], v[5]);
-    out[4 * t] = r.x; out[4 * t + 1] = r.y; out[4 * t + 2] = r.z; out[4 * t + 3] = r.w;
-}
-
-__global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
-{
-    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t < n) out[t] = dexp_dev(in[t]);
-}
-
-// ------------------------------------------------------------------------
 // Launchers
 // ------------------------------------------------------------------------
-static size_t eval_smem(const ChainDev& ch)
-{
-    if (ch.W <= 16) return (size_t)ch.po_bytes + 16 * (kEvalWarps + 1) + (size_t)kEvalWarps * 2 * 32 * (2 * ch.W) * 4;
-    return (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
-}
-
-template <int W>
-static void* eval_fn_w() { return (void*)eval_batch_w_kernel<W>; }
-
-static void* eval_pick(uint32_t W)
-{
-    switch (W) {
-    case 1: return eval_fn_w<1>();   case 2: return eval_fn_w<2>();   case 3: return eval_fn_w<3>();
-    case 4: return eval_fn_w<4>();   case 5: return eval_fn_w<5>();   case 6: return eval_fn_w<6>();
-    case 7: return eval_fn_w<7>();   case 8: return eval_fn_w<8>();   case 9: return eval_fn_w<9>();
-    case 10: return eval_fn_w<10>(); case 11: return eval_fn_w<11>(); case 12: return eval_fn_w<12>();
-    case 13: return eval_fn_w<13>(); case 14: return eval_fn_w<14>(); case 15: return eval_fn_w<15>();
-    case 16: return eval_fn_w<16>();
-    default: return (void*)eval_batch_kernel;
-    }
-}
-
-cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out, cudaStream_t st,
-                              int num_sms, uint64_t* launches)
-{
-    if (n_cand == 0) return cudaSuccess;
-    const size_t sm = eval_smem(ch);
-    void* fn = eval_pick(ch.W);
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    if (e != cudaSuccess) return e;
-    int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kEvalWarps * 32, sm);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-    const uint64_t tiles = (n_cand + 31) / 32;
-    uint64_t grid = (uint64_t)per_sm * num_sms;
-    const uint64_t need = (tiles + kEvalWarps - 1) / kEvalWarps;
-    if (grid > need) grid = need;
-    ChainDev c = ch;
-    const uint64_t* b = bits;
-    double* o = out;
-    void* args[] = {&c, &b, &n_cand, &o};
-    e = cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kEvalWarps * 32), args, sm, st);
-    if (launches) ++*launches;
-    return e;
-}
-
 size_t ga_smem_bytes(const GaArgs& a) { return smem_layout(a, nullptr, nullptr); }
 
 template <int WT>
@@ -1866,30 +1297,6 @@ cudaError_t launch_ga(const GaArgs& a, int grid, cudaStream_t st, uint64_t* laun
     e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, ga_smem_bytes(a), st);
     if (launches) ++*launches;
     return e;
-}
-
-cudaError_t launch_eval_stats(const ChainDev& ch, const uint64_t* bits, int64_t* stats_out, double* f_out,
-                              cudaStream_t st)
-{
-    const size_t sm = (size_t)(ch.p_words + ch.o_words) * 4 + 16;
-    cudaError_t e = cudaFuncSetAttribute(eval_stats_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    if (e != cudaSuccess) return e;
-    eval_stats_kernel<<<1, 32, sm, st>>>(ch, bits, stats_out, f_out);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_selftest_philox(const uint32_t* in, uint32_t n, uint32_t* out, cudaStream_t st)
-{
-    if (n == 0) return cudaSuccess;
-    selftest_philox_kernel<<<(n + 127) / 128, 128, 0, st>>>(in, n, out);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_selftest_dexp(const double* in, uint32_t n, double* out, cudaStream_t st)
-{
-    if (n == 0) return cudaSuccess;
-    selftest_dexp_kernel<<<(n + 127) / 128, 128, 0, st>>>(in, n, out);
-    return cudaGetLastError();
 }
 
 }  // namespace splitga

@@ -1,5 +1,5 @@
 // split_internal.h — device state and kernel launchers shared by split_host.cpp
-// and split_kernels.cu (product code; nothing here is shared with oracle/).
+// and the kernel units split_eval.cu / split_ga.cu (product code; nothing here is shared with oracle/).
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -84,7 +84,7 @@ struct GaArgs {
     uint32_t trace_gens;
 };
 
-// Launchers (split_kernels.cu).  Return cudaError_t of the launch.
+// Launchers (split_eval.cu, split_ga.cu).  Return cudaError_t of the launch.
 cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out,
                               cudaStream_t st, int num_sms, uint64_t* launches);
 // Cooperative persistent GA kernel; grid = blocks_per_sm * num_sms.
