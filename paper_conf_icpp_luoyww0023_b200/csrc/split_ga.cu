@@ -25,21 +25,25 @@ __device__ __forceinline__ void row_store(const Row<WT>& r, uint64_t* dst, uint3
     for (int i = 0; i < WT; ++i)
         if (i < (int)W) dst[i] = r.w[i];
 }
+// Row words are selected with arithmetic masks, never with a runtime index: an
+// indexed access would move the whole row to local memory (ptxas does that to
+// if-chains over a runtime word index).
 template <int WT>
 __device__ __forceinline__ void row_xor_bit(Row<WT>& r, uint32_t p)
 {
+    const uint32_t wi = p >> 6;
+    const uint64_t bit = 1ull << (p & 63);
 #pragma unroll
-    for (int i = 0; i < WT; ++i)
-        if ((uint32_t)i == (p >> 6)) r.w[i] ^= 1ull << (p & 63);
+    for (int i = 0; i < WT; ++i) r.w[i] ^= bit & (0ull - (uint64_t)((uint32_t)i == wi));
 }
 template <int WT>
 __device__ __forceinline__ bool row_get_bit(const Row<WT>& r, uint32_t p)
 {
-    bool b = false;
+    const uint32_t wi = p >> 6;
+    uint64_t b = 0;
 #pragma unroll
-    for (int i = 0; i < WT; ++i)
-        if ((uint32_t)i == (p >> 6)) b = (r.w[i] >> (p & 63)) & 1ull;
-    return b;
+    for (int i = 0; i < WT; ++i) b |= r.w[i] & (0ull - (uint64_t)((uint32_t)i == wi));
+    return (b >> (p & 63)) & 1ull;
 }
 __device__ __forceinline__ uint64_t word_mask(const ChainDev& ch, uint32_t w)
 {
@@ -74,26 +78,89 @@ __device__ __forceinline__ uint32_t select_bit(uint64_t m, uint32_t r)
 template <int WT>
 __device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch, uint32_t r, bool among_set)
 {
-    bool done = false;
+    // find the word holding the r-th candidate position, then toggle it with a mask
+    uint32_t wi = 0xFFFFFFFFu, rr = 0;
+    uint64_t mw = 0;
 #pragma unroll
     for (int i = 0; i < WT; ++i) {
-        if (i < (int)ch.W && !done) {
+        if (i < (int)ch.W) {
             const uint64_t m = (among_set ? row.w[i] : ~row.w[i]) & word_mask(ch, i);
             const uint32_t c = __popcll(m);
-            if (r < c) {
-                row.w[i] ^= 1ull << select_bit(m, r);
-                done = true;
-            } else {
-                r -= c;
-            }
+            const bool here = (wi == 0xFFFFFFFFu) && r < c;
+            wi = here ? (uint32_t)i : wi;
+            mw = here ? m : mw;
+            rr = here ? r : rr;
+            r -= (wi == 0xFFFFFFFFu) ? c : 0u;
         }
     }
+    const uint64_t bit = 1ull << select_bit(mw, rr);
+#pragma unroll
+    for (int i = 0; i < WT; ++i) row.w[i] ^= bit & (0ull - (uint64_t)((uint32_t)i == wi));
+}
+
+// Narrow rows (W <= 4): one loop iteration per cut, descending, over the
+// row's 32-bit halves held in registers (the next non-empty half is chosen
+// from an occupancy mask with a select tree, never with a runtime index), so
+// the trip count is the child's cut count rather than a per-word maximum.
+// Same integer statistics and Eq. 2 tail as eval_walk (R3, R5').
+template <int WT>
+__device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
+                                                   const Row<WT>& r)
+{
+    constexpr int NH = 2 * WT;
+    uint32_t h[NH];
+    uint32_t occ = 0, cuts = 0;
+#pragma unroll
+    for (int i = 0; i < NH; ++i) {
+        const uint64_t wv = (i / 2 < (int)ch.W) ? (r.w[i / 2] & word_mask(ch, i / 2)) : 0ull;
+        h[i] = (uint32_t)(wv >> (32 * (i & 1)));
+        occ |= (h[i] != 0u ? 1u : 0u) << i;
+        cuts += __popc(h[i]);
+    }
+    const uint32_t k = cuts + 1;
+    if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
+    uint32_t endP = ch.T, OV = 0, v = 0, qb = 0;
+    uint64_t S2 = 0;
+    for (uint32_t j = 0; j < cuts; ++j) {
+        if (v == 0u) {
+            const uint32_t q = bfind32(occ);
+            occ ^= 1u << q;
+            // select tree over the halves by the bits of q
+            uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
+#pragma unroll
+            for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
+            if constexpr (NH == 2) v = t1[0];
+            else if constexpr (NH == 4) v = (q & 2u) ? t1[1] : t1[0];
+            else {
+                const uint32_t a0 = (q & 2u) ? t1[1] : t1[0];
+                const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
+                v = (q & 4u) ? a1 : a0;
+            }
+            qb = q << 5;
+        }
+        const uint32_t bt = bfind32(v);
+        v ^= 1u << bt;
+        const uint32_t p = qb + bt;
+        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+        const uint32_t Pp = sP[p + 1], op = sO[p];
+        const uint32_t t = endP - Pp + op;
+        S2 += (uint64_t)t * t;
+        OV += op;
+        endP = Pp;
+    }
+    S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
+    const uint64_t S1 = (uint64_t)ch.T + OV;
+    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+    return eq2(k, V, OV, ch.T);
 }
 
 template <int WT>
 __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
                                             const Row<WT>& r, Stats* st)
 {
+    if constexpr (WT <= 4) {
+        if (!st) return eval_regs_narrow<WT>(ch, sP, sO, r);
+    }
     // same arithmetic as eval_walk, with the word loop unrolled over the register row
     uint32_t cuts = 0;
 #pragma unroll
@@ -837,7 +904,7 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
 // ------------------------------------------------------------------------
 template <int WT>
 __device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, uint32_t g, const double* fit,
-                                               const uint4& first)
+                                               const uint4& first, const double* fpre)
 {
     uint32_t best = 0;
     double bf = 0.0;
@@ -848,7 +915,7 @@ __device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, ui
 #pragma unroll
         for (int l = 0; l < 4; ++l) {
             ids[l] = below(lane_of(r, l), a.N);
-            fs[l] = (d + l < a.s) ? __ldcg(fit + ids[l]) : 0.0;
+            fs[l] = (d + l < a.s) ? ((d == 0 && fpre) ? fpre[l] : __ldcg(fit + ids[l])) : 0.0;
         }
 #pragma unroll
         for (int l = 0; l < 4; ++l) {
@@ -937,7 +1004,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
                                                double* fitn, const uint32_t* sP, const uint32_t* sO,
                                                const uint64_t* tau_ptr, uint32_t* s_ccnt, uint64_t* ckey,
                                                uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx,
-                                               const BestRow<WT>& snap, ChildDraws& pre, bool& have_pre)
+                                               const BestRow<WT>& snap, ChildDraws& pre, bool& have_pre,
+                                               const double* fpre)
 {
     const ChainDev& ch = a.ch;
     const uint32_t W = ch.W, N = a.N, E = a.E;
@@ -957,7 +1025,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         ChildDraws dr;
         if (cidx_ == first && have_pre) dr = pre;
         else dr = child_draws(a, gid, h, g);
-        const uint32_t mine = valid ? tournament<WT>(a, gid, g, fitc, dr.sel) : 0u;     // a4
+        const uint32_t mine =
+            valid ? tournament<WT>(a, gid, g, fitc, dr.sel, (cidx_ == first && have_pre) ? fpre : nullptr) : 0u;   // a4
         const uint32_t other = __shfl_xor_sync(0xFFFFFFFFu, mine, 1);
         if (tr) a.trace[(g - a.g_begin) * 16 + 8] = gtimer() + 0 * mine;
         if (!valid) continue;
@@ -1158,6 +1227,8 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
     uint32_t mph = 0;
     ChildDraws pre;
     bool have_pre = false;
+    double fpre[4];                   // prefetched fitness of the first tournament (s <= 4)
+    bool have_fpre = false;
     unsigned int bar_target = 0;      // generation barrier counter (zeroed by the host per launch)
     BestRow<WT> snap;
     snap.f = -CUDART_INF;         // first phase of a launch: no filter (all children compared)
@@ -1208,19 +1279,24 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             breed_children<WT>(a, i, g, my_local, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * Ns,
                                a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
                                a.tau + tau_par * I + i, sm.misc + 24, a.cand_key[Lb] + reg, a.cand_idx[Lb] + reg,
-                               a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre);
+                               a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre,
+                               have_fpre ? fpre : nullptr);
             // snapshot for breed(g+1), read before the barrier: REC(g-1) (parity of g+1),
             // stable during this phase and a lower bound of every later record
             snap = load_snapshot<WT>(a, i, nxt);
-            __syncthreads();
-            if (threadIdx.x == 0) {
-                a.cand_cnt[((size_t)Lb * I + i) * cpp + my_local] = sm.misc[24];    // publish, reset
-                sm.misc[24] = 0;
-            }
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
         }
-        gbar_arrive(a.gbar);
+        // arrive: the CTA barrier of the arrival also orders this CTA's candidate
+        // appends before thread 0 publishes their count (released with the arrival)
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (worker) {
+                a.cand_cnt[((size_t)Lb * I + my_island) * cpp + my_local] = sm.misc[24];
+                sm.misc[24] = 0;
+            }
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(a.gbar) : "memory");
+        }
         if (worker) precompute_draws(a, my_island, g, my_local, pre, have_pre);
         bar_target += gridDim.x;
         gbar_wait(a.gbar, bar_target);
@@ -1229,8 +1305,20 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             if (blockIdx.x == I) a.trace[(g - a.g_begin) * 16 + 7] = gtimer();
         }
         if (g == a.g_begin && blockIdx.x == 0 && threadIdx.x == 0) a.ctl->full = 0;   // every CTA read it earlier
-        if (__ldcg(&a.ctl->done)) break;
-        if (__ldcg(&a.ctl->redo[cur]) == g + 1) {
+        // one L2 round trip after the barrier: the stop / redo flags and the first
+        // tournament's fitness gathers of generation g+1 are issued together
+        have_fpre = false;
+        if (worker && have_pre && a.s <= 4) {
+            const double* fitq = a.fit[nxt] + (size_t)my_island * Ns;
+#pragma unroll
+            for (uint32_t l = 0; l < 4; ++l) fpre[l] = (l < a.s) ? __ldcg(fitq + below(lane_of(pre.sel, l), N)) : 0.0;
+            have_fpre = true;
+        }
+        const uint32_t done_f = __ldcg(&a.ctl->done);
+        const uint32_t redo_f = __ldcg(&a.ctl->redo[cur]);
+        if (done_f) break;
+        if (redo_f == g + 1) {
+            have_fpre = false;                // the exact top-E rewrites elite slots of g+1
             // a candidate list overflowed: exact top-E of generation g (still intact)
             general_select(a, a.fit[cur], E, false, sm, grid);
             if (is_leader) {

@@ -1,0 +1,56 @@
+"""Per-phase timing of the GA kernel's generation loop (C2), from the
+%globaltimer probes compiled in with SPLIT_TRACE_BUILD=1 (tuning only: the
+product build has none).  Usage on a GPU box:
+    SPLIT_TRACE_BUILD=1 python -m paper_conf_icpp_luoyww0023_b200.build --force
+    SPLIT_TRACE=gpurun_out/trace.csv python tools/trace_ga.py run
+and here:  python tools/trace_ga.py show gpurun_out/trace.csv"""
+import csv
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+
+def run():
+    import torch
+    from paper_conf_icpp_luoyww0023_b200 import split as S
+    from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+    torch.cuda.set_device(0)
+    lat, ovh = wl.chain("resnet50_175")
+    h = S.SplitGA(lat, ovh, pop_size=65536, n_elite=1024, k_min=2, k_max=32, stream=torch.cuda.current_stream())
+    for seed in range(3):
+        r = h.run(500, seed)
+    print(r["fitness"])
+    h.close()
+
+
+def show(path):
+    rows = list(csv.DictReader(open(path)))
+    rows = [r for r in rows if int(r["work_start"]) and int(r["work_sync"])]
+    pairs = [("work_start", "b_tourn", "tournament (fitness gathers)"),
+             ("b_tourn", "b_rows", "parent rows"),
+             ("b_rows", "b_xover", "crossover"),
+             ("b_xover", "b_repair", "mutate + repair"),
+             ("b_repair", "b_eval", "fused eval"),
+             ("b_eval", "b_cand", "store + candidate append"),
+             ("b_cand", "b_rec", "record filter"),
+             ("b_rec", "work_end", "snapshot + CTA sync"),
+             ("work_end", "work_sync", "grid barrier (worker)"),
+             ("lead_start", "lead_loaded", "leader: TMA loads"),
+             ("lead_loaded", "lead_record", "leader: record"),
+             ("lead_record", "lead_sort", "leader: gather + sort"),
+             ("lead_sort", "lead_end", "leader: merge + copy"),
+             ("lead_end", "lead_sync", "grid barrier (leader)")]
+    for a, b, name in pairs:
+        d = sorted(int(r[b]) - int(r[a]) for r in rows if int(r[a]) and int(r[b]))
+        if d:
+            print(f"{name:32s} median {d[len(d) // 2] / 1e3:7.2f} us   p90 {d[int(len(d) * 0.9)] / 1e3:7.2f} us")
+    per = sorted(int(rows[i + 1]["work_sync"]) - int(rows[i]["work_sync"]) for i in range(len(rows) - 1))
+    print(f"{'generation (worker sync to sync)':32s} median {per[len(per) // 2] / 1e3:7.2f} us")
+
+
+if __name__ == "__main__":
+    if sys.argv[1] == "run":
+        run()
+    else:
+        show(sys.argv[2])
