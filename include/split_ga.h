@@ -157,6 +157,30 @@ int split_comm_unique_id(uint8_t out[128]);
 int split_comm_init(const uint8_t id[128], int rank, int world, int device, void** comm);
 void split_comm_destroy(void* comm);
 
+/* f1 — exact optimum by exhaustive enumeration of all 2^(n_ops-1) splits
+ * (the quantity the GA approximates, P@9901-10019 counts
+ * 287,980 profiled candidates for 3 cuts of ResNet50).  Requires
+ * n_ops - 1 <= 44 and k_max <= 64 (SPLIT_E_INVAL otherwise); the time grows as
+ * 2^(n_ops-1) (about 2^40 splits per second on one B200).  best_out receives
+ * the canonical best (fitness desc, bitset asc; R10) over k in [k_min, k_max]
+ * with its statistics (evaluations = 2^(n_ops-1), generation fields 0);
+ * best_out->bits: host buffer of split_words() words.  If min_v_per_k (host,
+ * k_max+1 entries) is non-NULL it receives the minimum V = k*S2 - S1^2 over all
+ * splits with k blocks (-1 where none), for k in [0, k_max]; argmin_per_k
+ * (host, k_max+1) the smallest bitset attaining it.  Synchronous, on the
+ * handle's stream; device scratch is allocated and freed inside the call. */
+int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* min_v_per_k, uint64_t* argmin_per_k);
+
+/* f1 — minimum S2 = sum t_j^2 over all k-block splits, k = 1..k_max, by the
+ * O(k n^2) dynamic program D[j][i] = min_p D[j-1][p] + (P[i]-P[p]+ovh[p-1])^2
+ * (one CTA on the handle's device).  Exact for any per-cut overheads; with a
+ * constant overhead delta, S1 = T + (k-1) delta is fixed and
+ * V*_k = k*S2*_k - S1^2 is the minimum variance.  s2_out: host,
+ * k_max+1 entries ([0] = UINT64_MAX; UINT64_MAX where k > n_ops).
+ * 1 <= k_max <= the handle's k_max (the create-time guard keeps every sum in
+ * range).  Synchronous. */
+int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out);
+
 void split_ga_destroy(split_ga_t* h);
 const char* split_strerror(int code);
 const char* split_last_error(void);

@@ -167,6 +167,9 @@ struct split_ga_t {
     cudaEvent_t ev[4];
     unsigned long long* d_trace;   // SPLIT_TRACE=<csv path>: phase timestamps of the first RUN segment
     uint32_t trace_gens;
+    // host copy of the chain words: P[0..n] | ovh[0..n-2] (f1 exact solvers)
+    std::vector<uint32_t> hwords;
+    uint32_t p_words;
     // eval_batch_host staging
     uint64_t* d_hbits[2];
     double* d_hfit[2];
@@ -349,6 +352,8 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
             return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
         }
     }
+    h->hwords = words;
+    h->p_words = p_words;
     ChainDev& ch = h->ch;
     ch.po = (const uint2*)d_po;
     ch.po_bytes = (uint32_t)(po.size() * 4);
@@ -807,5 +812,164 @@ extern "C" int split_selftest_dexp(int device, const double* in, uint32_t n, dou
     cudaFree(di);
     cudaFree(dout);
     if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "selftest_dexp: %s", cudaGetErrorString(e));
+    return SPLIT_OK;
+}
+
+// ------------------------------------------------------------------------
+// f1 exact solvers: exhaustive enumeration and the DP
+// ------------------------------------------------------------------------
+#define RC(x)                      \
+    do {                            \
+        const int rc_ = (x);        \
+        if (rc_ != SPLIT_OK) return rc_; \
+    } while (0)
+
+namespace {
+// scratch owned by one call (freed on every exit path)
+struct DevScratch {
+    std::vector<void*> p;
+    ~DevScratch()
+    {
+        for (void* q : p) cudaFree(q);
+    }
+    template <class T>
+    int alloc(T** out, size_t count)
+    {
+        void* q = nullptr;
+        cudaError_t e = cudaMalloc(&q, count * sizeof(T) + 16);
+        if (e != cudaSuccess) return fail(SPLIT_E_NOMEM, "cudaMalloc(%zu): %s", count * sizeof(T), cudaGetErrorString(e));
+        p.push_back(q);
+        *out = (T*)q;
+        return SPLIT_OK;
+    }
+};
+}  // namespace
+
+extern "C" int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* min_v_per_k, uint64_t* argmin_per_k)
+{
+    if (!h || !best_out || !best_out->bits) return fail(SPLIT_E_INVAL, "split_exhaustive: NULL argument");
+    const uint32_t m = h->n - 1;
+    if (m > kExhMaxPos) return fail(SPLIT_E_INVAL, "split_exhaustive: n_ops - 1 = %u cut positions > %u", m, kExhMaxPos);
+    if (h->p.k_max > 64) return fail(SPLIT_E_INVAL, "split_exhaustive: k_max must be <= 64");
+    CU(cudaSetDevice(h->device));
+    const uint32_t c = m < kExhLow ? m : kExhLow;
+    // A[p] = P[p+1] (A[m] = T), B[p] = P[p+1] - ovh[p] (mod 2^32)
+    std::vector<uint32_t> A(m + 1), B(m > 0 ? m : 1);
+    for (uint32_t q = 0; q <= m; ++q) A[q] = h->hwords[q + 1];
+    for (uint32_t q = 0; q < m; ++q) B[q] = h->hwords[q + 1] - h->hwords[h->p_words + q];
+    DevScratch sc;
+    uint32_t *dA, *dB;
+    void *dtab, *dres, *dout;
+    uint64_t *dkv, *dkv2;
+    const size_t rows = m - c + 1, nb = (size_t)1 << c;
+    RC(sc.alloc(&dA, A.size()));
+    RC(sc.alloc(&dB, B.size()));
+    RC(sc.alloc((uint8_t**)&dtab, rows * nb * 16));
+    RC(sc.alloc(&dkv, 65));
+    RC(sc.alloc(&dkv2, 65));
+    CU(cudaMemcpyAsync(dA, A.data(), A.size() * 4, cudaMemcpyHostToDevice, h->stream));
+    CU(cudaMemcpyAsync(dB, B.data(), B.size() * 4, cudaMemcpyHostToDevice, h->stream));
+    ExhArgs a;
+    memset(&a, 0, sizeof(a));
+    a.A = dA;
+    a.B = dB;
+    a.tab = dtab;
+    a.m = m;
+    a.c = c;
+    a.T = (uint32_t)h->T;
+    a.k_min = h->p.k_min;
+    a.k_max = h->p.k_max;
+    a.outer_total = (uint64_t)1 << (m - c);
+    a.seed_f = 0.0;
+    // grid: enough threads to fill every SM, each walking a contiguous Gray range
+    const uint64_t max_threads = (uint64_t)exh_blocks_per_sm(a) * h->num_sms * kExhThreads;
+    uint64_t threads = a.outer_total < max_threads ? a.outer_total : max_threads;
+    a.per_thread = (a.outer_total + threads - 1) / threads;
+    threads = (a.outer_total + a.per_thread - 1) / a.per_thread;
+    const uint32_t grid = (uint32_t)((threads + kExhThreads - 1) / kExhThreads);
+    RC(sc.alloc((uint8_t**)&dres, (size_t)grid * 16));
+    RC(sc.alloc((uint8_t**)&dout, 16));
+    a.res = dres;
+    h->stats.launches = 0;
+    CU(launch_exh_table(a, h->stream));
+    ++h->stats.launches;
+    CU(cudaEventRecord(h->ev[0], h->stream));
+    CU(launch_exh(a, MODE_EXH_BEST, grid, h->stream));
+    CU(launch_exh_reduce(dres, grid, dout, h->stream));
+    CU(cudaEventRecord(h->ev[2], h->stream));
+    h->stats.launches += 2;
+    struct {
+        double f;
+        uint64_t bits;
+    } best;
+    CU(cudaMemcpyAsync(&best, dout, 16, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    CU(cudaEventElapsedTime(&h->stats.ms_total, h->ev[0], h->ev[2]));
+    h->stats.ms_loop = h->stats.ms_total;
+    if (best.f == -INFINITY) return fail(SPLIT_E_STATE, "split_exhaustive: no split with k in [k_min, k_max]");
+    // statistics of the best split (same kernel as split_ga_run's)
+    CU(cudaMemcpyAsync(h->d_bits1, &best.bits, 8, cudaMemcpyHostToDevice, h->stream));
+    CU(launch_eval_stats(h->ch, h->d_bits1, h->d_stats, h->d_statf, h->stream));
+    ++h->stats.launches;
+    int64_t st[5];
+    double fchk;
+    CU(cudaMemcpyAsync(st, h->d_stats, sizeof(st), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaMemcpyAsync(&fchk, h->d_statf, 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    if (fchk != best.f) return fail(SPLIT_E_STATE, "split_exhaustive: best fitness mismatch (internal)");
+    best_out->bits[0] = best.bits;
+    for (uint32_t w = 1; w < h->W; ++w) best_out->bits[w] = 0;
+    best_out->fitness = best.f;
+    best_out->k = (uint32_t)st[0];
+    best_out->var_num = st[1];
+    best_out->s1 = (uint64_t)st[2];
+    best_out->s2 = (uint64_t)st[3];
+    best_out->overhead_ns = (uint64_t)st[4];
+    best_out->expected_wait_ns = st[2] > 0 ? (double)(uint64_t)st[3] / (2.0 * (double)(uint64_t)st[2]) : 0.0;
+    best_out->generation_found = 0;
+    best_out->generations_run = 0;
+    best_out->evaluations = (uint64_t)1 << m;
+    if (min_v_per_k || argmin_per_k) {
+        // MINV pass: min V per k <= k_max; ARGMIN pass: smallest bitset attaining it
+        std::vector<uint64_t> init(65, ~0ull), kv(65), kb(65);
+        CU(cudaMemcpyAsync(dkv, init.data(), 65 * 8, cudaMemcpyHostToDevice, h->stream));
+        a.kv_out = dkv;
+        CU(launch_exh(a, MODE_EXH_MINV, grid, h->stream));
+        ++h->stats.launches;
+        CU(cudaMemcpyAsync(kv.data(), dkv, 65 * 8, cudaMemcpyDeviceToHost, h->stream));
+        if (argmin_per_k) {
+            CU(cudaMemcpyAsync(dkv2, init.data(), 65 * 8, cudaMemcpyHostToDevice, h->stream));
+            a.kv = dkv;
+            a.kv_out = dkv2;
+            CU(launch_exh(a, MODE_EXH_ARGMIN, grid, h->stream));
+            ++h->stats.launches;
+            CU(cudaMemcpyAsync(kb.data(), dkv2, 65 * 8, cudaMemcpyDeviceToHost, h->stream));
+        }
+        CU(cudaStreamSynchronize(h->stream));
+        for (uint32_t k = 0; k <= h->p.k_max; ++k) {
+            if (min_v_per_k) min_v_per_k[k] = (kv[k] == ~0ull) ? -1 : (int64_t)kv[k];
+            if (argmin_per_k) argmin_per_k[k] = (kv[k] == ~0ull) ? 0 : kb[k];
+        }
+    }
+    return SPLIT_OK;
+}
+
+extern "C" int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out)
+{
+    if (!h || !s2_out) return fail(SPLIT_E_INVAL, "split_dp_min_s2: NULL argument");
+    if (k_max < 1 || k_max > h->p.k_max)
+        return fail(SPLIT_E_INVAL, "split_dp_min_s2: k_max must be in [1, handle k_max = %u]", h->p.k_max);
+    CU(cudaSetDevice(h->device));
+    DevScratch sc;
+    uint64_t* d_out;
+    RC(sc.alloc(&d_out, (size_t)k_max + 1));
+    CU(cudaEventRecord(h->ev[0], h->stream));
+    CU(launch_dp(h->ch.words, h->ch.words + h->ch.p_words, h->n, k_max, d_out, h->stream));
+    CU(cudaEventRecord(h->ev[2], h->stream));
+    h->stats.launches = 1;
+    CU(cudaMemcpyAsync(s2_out, d_out, ((size_t)k_max + 1) * 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    CU(cudaEventElapsedTime(&h->stats.ms_total, h->ev[0], h->ev[2]));
+    h->stats.ms_loop = h->stats.ms_total;
     return SPLIT_OK;
 }

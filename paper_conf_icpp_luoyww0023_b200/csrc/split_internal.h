@@ -84,6 +84,33 @@ struct GaArgs {
     uint32_t trace_gens;
 };
 
+// f1 exact solvers (split_exact.cu)
+enum ExhMode : int { MODE_EXH_BEST = 0, MODE_EXH_MINV = 1, MODE_EXH_ARGMIN = 2 };
+constexpr uint32_t kExhThreads = 256;   // threads per CTA of the enumeration kernel
+constexpr uint32_t kExhQ = 64;          // survivor queue entries per warp (>= 63)
+constexpr uint32_t kExhLow = 6;         // low cut positions served by the (H, Bl) table
+constexpr uint32_t kExhMaxPos = 44;     // n_ops - 1 <= 44 cut positions (2^44 splits)
+struct ExhArgs {
+    const uint32_t* A;     // [m+1] A[p] = P[p+1] (A[m] = T): end of a block closed by cut p
+    const uint32_t* B;     // [m]   B[p] = P[p+1] - ovh[p] (mod 2^32): start offset after cut p
+    void* tab;             // [(m-c+1) << c] ExhEntry
+    uint32_t m, c;         // cut positions n-1, low positions
+    uint32_t T, k_min, k_max;
+    uint64_t outer_total;  // 2^(m-c) high-part states
+    uint64_t per_thread;   // high-part states per thread
+    void* res;             // [grid] per-CTA best (MODE_EXH_BEST)
+    const uint64_t* kv;    // [k_max+1] min V per k (input of MODE_EXH_ARGMIN)
+    uint64_t* kv_out;      // [k_max+1] min V (MINV) or argmin bitset (ARGMIN), atomicMin targets
+    double seed_f;         // a known fitness (< 0) to seed the filter, or 0
+};
+size_t exh_smem_bytes(const ExhArgs& a);
+int exh_blocks_per_sm(const ExhArgs& a);
+cudaError_t launch_exh_table(const ExhArgs& a, cudaStream_t st);
+cudaError_t launch_exh(const ExhArgs& a, int mode, uint32_t grid, cudaStream_t st);
+cudaError_t launch_exh_reduce(const void* res, uint32_t n, void* out, cudaStream_t st);
+cudaError_t launch_dp(const uint32_t* P, const uint32_t* ovh, uint32_t n, uint32_t k_max, uint64_t* s2_out,
+                      cudaStream_t st);
+
 // Launchers (split_eval.cu, split_ga.cu).  Return cudaError_t of the launch.
 cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t n_cand, double* out,
                               cudaStream_t st, int num_sms, uint64_t* launches);

@@ -85,6 +85,8 @@ def _load():
         "split_selftest_philox": (C.c_int, [C.c_int, C.c_void_p, C.c_uint32, C.c_void_p]),
         "split_selftest_dexp": (C.c_int, [C.c_int, C.c_void_p, C.c_uint32, C.c_void_p]),
         "split_last_run_stats": (C.c_int, [C.c_void_p, P(split_run_stats)]),
+        "split_exhaustive": (C.c_int, [C.c_void_p, P(split_best_t), C.c_void_p, C.c_void_p]),
+        "split_dp_min_s2": (C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -98,7 +100,7 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_eval_batch_host", "split_ga_run", "split_ga_population", "split_preempt_decide",
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
-            "split_last_run_stats")
+            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2")
 
 
 def lib():
@@ -224,6 +226,29 @@ class SplitGA:
         _check(_lib.split_ga_run(self._h, generations, seed, C.byref(best)), "split_ga_run")
         out = {f: getattr(best, f) for f, _ in split_best_t._fields_ if f != "bits"}
         out["bits"] = bits
+        return out
+
+    # f1: exact optimum over all 2^(n_ops-1) splits (and optionally min V / argmin per k)
+    def exhaustive(self, per_k: bool = False) -> dict:
+        bits = np.zeros(max(self.W, 1), dtype=np.uint64)
+        best = split_best_t()
+        best.bits = bits.ctypes.data_as(C.POINTER(C.c_uint64))
+        kmax = int(self.params.k_max)
+        mv = np.zeros(kmax + 1, dtype=np.int64) if per_k else None
+        am = np.zeros(kmax + 1, dtype=np.uint64) if per_k else None
+        _check(_lib.split_exhaustive(self._h, C.byref(best), _ptr(mv) if per_k else None,
+                                     _ptr(am) if per_k else None), "split_exhaustive")
+        out = {f: getattr(best, f) for f, _ in split_best_t._fields_ if f != "bits"}
+        out["bits"] = bits
+        if per_k:
+            out["min_v_per_k"] = mv
+            out["argmin_per_k"] = am
+        return out
+
+    # f1: min S2 per block count by the O(k n^2) DP
+    def dp_min_s2(self, k_max: int) -> np.ndarray:
+        out = np.zeros(k_max + 1, dtype=np.uint64)
+        _check(_lib.split_dp_min_s2(self._h, k_max, _ptr(out)), "split_dp_min_s2")
         return out
 
     def population(self, island: int = 0):
