@@ -35,6 +35,7 @@ C2 = dict(chain="resnet50_175", pop_size=65536, n_elite=1024, tournament_size=4,
           p_mutation=0.2, k_min=2, k_max=32, generations=500)
 MIGRATION_INTERVAL, N_MIGRANTS = 10, 64
 C5_EVAL_N = 1 << 24           # split_eval_batch sub-measurement (C5: n = 1024, 2.3 GB of bitsets > L2)
+EXACT_N = 33                  # f1 sub-measurement: split_exhaustive over 2^32 splits
 CPU_SAMPLE_GENERATIONS = 100  # oracle cpu_baseline: about 10 s of one core
 REF_STEP_GENERATIONS = 10     # --impl reference: oracle generations per step
 
@@ -199,6 +200,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-eval", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-exact", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
@@ -294,6 +296,26 @@ def main():
         "roofline": roofline,
     }
 
+    # e2e through the public API with host buffers: create (H2D of the chain) + run + best (D2H)
+    if not args.no_e2e:
+        e2e_steps = max(3, min(args.steps, 10))
+        e_evals = 0
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for i in range(e2e_steps):
+            with S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl) as he:
+                e_evals += he.run(G, 5000 + i)["evaluations"]
+        torch.cuda.synchronize()
+        barrier()
+        et_s, ee_all, _ = D.reduce_max_sum(time.perf_counter() - t0, float(e_evals), device=dev)
+        n = len(lat)
+        h2d = 4 * (((n + 1 + 3) & ~3) + ((n - 1 + 3) & ~3)) + 8   # staged chain words + best bits
+        d2h = 48 + world * (W + 2) * 8 + 5 * 8 + 8                # control block, island records, best stats
+        out["e2e"] = {"value": ee_all / et_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
+                      "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+                      "note": "split_ga_create(host latencies) + split_ga_run + best to host + destroy, wall clock"}
+
     # split_eval_batch at C5 (HBM-bound; the north-star's >= 60 % target)
     if not args.no_eval:
         lat5, ovh5 = wl.chain("synthetic_1024")
@@ -326,25 +348,22 @@ def main():
         h5.close()
         del bits, fout
 
-    # e2e through the public API with host buffers: create (H2D of the chain) + run + best (D2H)
-    if not args.no_e2e:
-        e2e_steps = max(3, min(args.steps, 10))
-        e_evals = 0
-        barrier()
-        torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        for i in range(e2e_steps):
-            with S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl) as he:
-                e_evals += he.run(G, 5000 + i)["evaluations"]
-        torch.cuda.synchronize()
-        barrier()
-        et_s, ee_all, _ = D.reduce_max_sum(time.perf_counter() - t0, float(e_evals), device=dev)
-        n = len(lat)
-        h2d = 4 * (((n + 1 + 3) & ~3) + ((n - 1 + 3) & ~3)) + 8   # staged chain words + best bits
-        d2h = 48 + world * (W + 2) * 8 + 5 * 8 + 8                # control block, island records, best stats
-        out["e2e"] = {"value": ee_all / et_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
-                      "d2h_bytes_per_step": d2h, "steps": e2e_steps,
-                      "note": "split_ga_create(host latencies) + split_ga_run + best to host + destroy, wall clock"}
+    # f1 exact solver: exhaustive enumeration of all 2^32 splits of a 33-op chain
+    if not args.no_exact:
+        latx, ovhx = wl.random_chain(EXACT_N, 3, ovh_hi=100_000)
+        with S.SplitGA(latx, ovhx, pop_size=4, n_elite=0, k_min=2, k_max=32, device=local, stream=stream) as hx:
+            hx.exhaustive()
+            xm = []
+            for i in range(3):
+                rx = hx.exhaustive()
+                xm.append(hx.last_run_stats()["ms_total"])
+            s2 = hx.dp_min_s2(32)
+            dp_ms = hx.last_run_stats()["ms_total"]
+        xms = sum(xm) / len(xm)
+        out["exact"] = {"workload": f"f1: all 2^{EXACT_N - 1} splits of a {EXACT_N}-op synthetic chain, k in [2, 32]",
+                        "splits_per_s": (2 ** (EXACT_N - 1)) / (xms / 1000.0), "ms": xms,
+                        "best": {"fitness": rx["fitness"], "k": rx["k"]},
+                        "dp_ms_k32": dp_ms}
 
     out["clocks"] = clk.summary()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

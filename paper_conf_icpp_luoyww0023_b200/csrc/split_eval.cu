@@ -139,7 +139,7 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
 }
 
 template <int W, int NW_, int RPT_, int NB_>
-__global__ void __launch_bounds__(NW_ * 32) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
+__global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / NW_ : 1)) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
                                                                 uint64_t n_cand, double* __restrict__ out)
 {
     using Cfg = EvalCfg<W, NW_, RPT_, NB_>;
@@ -338,7 +338,7 @@ static size_t eval_smem_of(const ChainDev& ch, const EvalVariant& v)
 template <int W>
 static EvalVariant eval_default()
 {
-    if constexpr (W >= 12) return eval_variant<W, 8, 1, 1>();
+    if constexpr (W >= 12) return eval_variant<W, 15, 1, 1>();
     else if constexpr (W >= 6) return eval_variant<W, 8, 2, 1>();
     else return eval_variant<W, 8, 2, 2>();
 }
@@ -358,6 +358,9 @@ static EvalVariant eval_pick(uint32_t W)
         case 4: return eval_variant<16, 6, 2, 1>();
         case 5: return eval_variant<16, 8, 1, 2>();
         case 6: return eval_variant<16, 16, 1, 1>();
+        case 7: return eval_variant<16, 15, 1, 1>();
+        case 8: return eval_variant<16, 24, 1, 1>();
+        case 9: return eval_variant<16, 12, 1, 1>();
         default: break;
         }
     }
