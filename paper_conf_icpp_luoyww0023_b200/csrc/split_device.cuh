@@ -102,15 +102,39 @@ __device__ __forceinline__ double dexp_dev(double z)
     return __dmul_rn(__dmul_rn(p, s1), s2);
 }
 
+// RN(a/b) for a >= 0, b > 0 (no overflow or underflow) from rb = RN(1/b), in
+// five FP64 operations instead of the DDIV sequence.  q0 = RN(a rb) is within
+// ~2^-52 relative of a/b; one Newton correction (r = a - b q exactly-enough by
+// FMA) brings q within 1/2 ulp + O(2^-104), i.e. faithful; Markstein's theorem
+// (rb within 1/2 ulp of 1/b, q faithful => RN(q + (a - b q) rb) = RN(a/b), the
+// residual being exact) makes the second correction the correctly rounded
+// quotient -- the same value as the oracle's IEEE division (R5').
+__device__ __forceinline__ double div_rcp_rn(double a, double b, double rb)
+{
+    double q = __dmul_rn(a, rb);
+    double r = __fma_rn(-b, q, a);
+    q = __fma_rn(r, rb, q);
+    r = __fma_rn(-b, q, a);
+    return __fma_rn(r, rb, q);
+}
+
 // Eq. 2 from the exact integer statistics (R5'):
 //   x = sigma/T = sqrt(V)/(k T),  y = overhead/m = (OV/T)/k,  f = -(e^(x-1) + e^(y-1))
-__device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, uint32_t T)
+// rcp: ChainDev::rcp (rcp[0] = RN(1/T), rcp[k] = RN(1/k), rcp[n+1+k] = RN(1/(kT))).
+// k T < 2^37 is exact in FP64, so every quotient is the IEEE quotient of the
+// same operands the oracle divides.
+__device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, uint32_t T, uint32_t n, const double* rcp)
 {
+    const double rk = __ldg(rcp + k), rkT = __ldg(rcp + n + 1 + k), rT = __ldg(rcp);
     const double Td = __uint2double_rn(T);
     const double kd = __uint2double_rn(k);
-    const double x = __ddiv_rn(__dsqrt_rn(__ll2double_rn(V)), __dmul_rn(kd, Td));
-    const double y = __ddiv_rn(__ddiv_rn(__ull2double_rn(OV), Td), kd);
+    const double x = div_rcp_rn(__dsqrt_rn(__ll2double_rn(V)), __dmul_rn(kd, Td), rkT);
+    const double y = div_rcp_rn(div_rcp_rn(__ull2double_rn(OV), Td, rT), kd, rk);
     return -__dadd_rn(dexp_dev(__dsub_rn(x, 1.0)), dexp_dev(__dsub_rn(y, 1.0)));
+}
+__device__ __forceinline__ double eq2(uint32_t k, int64_t V, uint64_t OV, const ChainDev& ch)
+{
+    return eq2(k, V, OV, ch.T, ch.n, ch.rcp);
 }
 
 __device__ __forceinline__ unsigned long long gtimer()
@@ -231,6 +255,13 @@ __device__ __forceinline__ uint32_t opaque32(uint32_t x)
     asm volatile("mov.u32 %0, %0;" : "+r"(x));
     return x;
 }
+__device__ __forceinline__ uint2 lds64_if(bool pred, uint32_t a)
+{
+    uint2 v = make_uint2(0u, 0u);
+    asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p ld.shared.v2.u32 {%0, %1}, [%2]; }"
+                 : "+r"(v.x), "+r"(v.y) : "r"(a), "r"((uint32_t)pred));
+    return v;
+}
 __device__ __forceinline__ uint2 lds64(uint32_t a)
 {
     uint2 v;
@@ -348,7 +379,7 @@ __device__ __forceinline__ double eval_walk(const ChainDev& ch, const uint32_t* 
     S2 += (uint64_t)t * t;
     const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);   // exact: V < 2^63 by the a0 guard
     if (st) { st->k = k; st->V = V; st->S1 = S1; st->S2 = S2; st->OV = OV; }
-    return eq2(k, V, OV, ch.T);
+    return eq2(k, V, OV, ch);
 }
 
 }  // namespace splitga

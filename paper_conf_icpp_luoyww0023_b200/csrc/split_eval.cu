@@ -91,7 +91,9 @@ struct EvalCfg {
 };
 
 // occupancy mask of one row (bit q <=> half q non-empty, padding masked)
-template <int W>
+// EXACT: the sort key is the exact cut count (one POPC per half) instead of the
+// number of non-empty halves (always exact for W <= 4).
+template <int W, bool EXACT>
 __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, uint32_t validocc, uint32_t qfull,
                                                   uint32_t lastm, uint32_t& cuts)
 {
@@ -106,7 +108,7 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
             const uint4 v = my4[cc];
             cc = (cc + 1 == C) ? 0u : cc + 1;
             occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1) | (min(v.z, 1u) << 2) | (min(v.w, 1u) << 3)) << (4 * j);
-            if constexpr (W <= 4) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+            if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
         }
     } else {
         const uint2* my2 = (const uint2*)my;
@@ -116,7 +118,7 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
             const uint2 v = my2[cc];
             cc = (cc + 1 == W) ? 0u : cc + 1;
             occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1)) << (2 * j);
-            if constexpr (W <= 4) pc += __popc(v.x) + __popc(v.y);
+            if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y);
         }
     }
     // bit 4j+i (2j+i) of occr is half 4((j+l)%C)+i: rotate into place
@@ -124,7 +126,7 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
     uint32_t occ;
     if constexpr (H == 32) occ = __funnelshift_l(occr, occr, rot);
     else occ = ((occr << rot) | (occr >> ((H - rot) % H))) & ((1u << H) - 1u);
-    if constexpr (W <= 4) {
+    if constexpr (W <= 4 || EXACT) {
         // exact cut count (sort key); padding bits removed below
         for (uint32_t q = qfull; q < H; ++q) pc -= __popc(my[q] & ~((q == qfull) ? lastm : 0u));
     }
@@ -134,11 +136,11 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
         my[qfull] = vq;
         occ |= min(vq, 1u) << qfull;
     }
-    cuts = (W <= 4) ? pc : __popc(occ);
+    cuts = (W <= 4 || EXACT) ? pc : __popc(occ);
     return occ;
 }
 
-template <int W, int NW_, int RPT_, int NB_>
+template <int W, int NW_, int RPT_, int NB_, int KEY_ = 0>
 __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / NW_ : 1)) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
                                                                 uint64_t n_cand, double* __restrict__ out)
 {
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
             flags[h] = 0x4000u;                  // 0x4000: no row (ragged tail), 0x8000: k out of range
             if (row < rows) {
                 uint32_t cuts;
-                s_occ[row] = row_occupancy<W>(buf + row * H, lane, validocc, qfull, lastm, cuts);
+                s_occ[row] = row_occupancy<W, KEY_ != 0>(buf + row * H, lane, validocc, qfull, lastm, cuts);
                 const uint32_t ne = __popc(s_occ[row]);
                 // a row with >= k_max non-empty halves (or cuts) has k > k_max
                 flags[h] = (ne < ch.k_max && cuts < ch.k_max) ? 0u : 0x8000u;
@@ -236,41 +238,43 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
             if (pe & 0x4000u) continue;
             double f = -CUDART_INF;
             if (!(pe & 0x8000u)) {
-                uint32_t occ = s_occ[r];
-                uint32_t endP = ch.T, OV = 0, cnt = 0;
-                uint64_t S2 = 0;
-                const uint32_t my_s = smem_u32(buf + r * H);
-                uint32_t v = 0, tb = spo_s;      // current half's remaining bits and chain entries (spo + 32 q)
-                auto step = [&]() {
-                    // refill (predicated, no branch): next non-empty half when v is exhausted
-                    const uint32_t qn = bfind32(occ);
-                    const bool need = (v == 0u);
-                    if (need) occ ^= 1u << qn;
-                    v = lds32_if(need, my_s + 4u * qn, v);
-                    tb = need ? spo_s + (qn << 8) : tb;
-                    const uint32_t bt = bfind32(v);
-                    v ^= 1u << bt;
-                    // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
-                    const uint2 e = lds64(tb + 8u * bt);
-                    const uint32_t tj = endP - e.x + e.y;
-                    S2 += (uint64_t)tj * tj;
-                    OV += e.y;
-                    endP = e.x;
-                };
-                // unrolled by two (no register moves between iterations)
-                while (v | occ) {
-                    step();
-                    cnt += 1;
-                    if (!(v | occ)) break;
-                    step();
-                    cnt += 1;
-                }
-                const uint32_t k = cnt + 1;
-                if (k >= ch.k_min && k <= ch.k_max) {
-                    S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
-                    const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
-                    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
-                    f = eq2(k, V, OV, ch.T);
+                {
+                    uint32_t occ = s_occ[r];
+                    uint32_t endP = ch.T, OV = 0, cnt = 0;
+                    uint64_t S2 = 0;
+                    const uint32_t my_s = smem_u32(buf + r * H);
+                    uint32_t v = 0, tb = spo_s;      // current half's remaining bits and chain entries (spo + 32 q)
+                    auto step = [&]() {
+                        // refill (predicated, no branch): next non-empty half when v is exhausted
+                        const uint32_t qn = bfind32(occ);
+                        const bool need = (v == 0u);
+                        if (need) occ ^= 1u << qn;
+                        v = lds32_if(need, my_s + 4u * qn, v);
+                        tb = need ? spo_s + (qn << 8) : tb;
+                        const uint32_t bt = bfind32(v);
+                        v ^= 1u << bt;
+                        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+                        const uint2 e = lds64(tb + 8u * bt);
+                        const uint32_t tj = endP - e.x + e.y;
+                        S2 += (uint64_t)tj * tj;
+                        OV += e.y;
+                        endP = e.x;
+                    };
+                    // unrolled by two (no register moves between iterations)
+                    while (v | occ) {
+                        step();
+                        cnt += 1;
+                        if (!(v | occ)) break;
+                        step();
+                        cnt += 1;
+                    }
+                    const uint32_t k = cnt + 1;
+                    if (k >= ch.k_min && k <= ch.k_max) {
+                        S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
+                        const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
+                        const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+                        f = eq2(k, V, OV, ch);
+                    }
                 }
             }
             __stcs(out + row0 + r, f);
@@ -323,10 +327,11 @@ struct EvalVariant {
     uint32_t W, NW, RPT, NB;
 };
 
-template <int W, int NW, int RPT, int NB>
+template <int W, int NW, int RPT, int NB, int KEY = 0>
 static EvalVariant eval_variant()
 {
-    return EvalVariant{(void*)eval_batch_w_kernel<W, NW, RPT, NB>, (uint32_t)W, (uint32_t)NW, (uint32_t)RPT, (uint32_t)NB};
+    return EvalVariant{(void*)eval_batch_w_kernel<W, NW, RPT, NB, KEY>, (uint32_t)W, (uint32_t)NW, (uint32_t)RPT,
+                       (uint32_t)NB};
 }
 
 static size_t eval_smem_of(const ChainDev& ch, const EvalVariant& v)
@@ -361,6 +366,11 @@ static EvalVariant eval_pick(uint32_t W)
         case 7: return eval_variant<16, 15, 1, 1>();
         case 8: return eval_variant<16, 24, 1, 1>();
         case 9: return eval_variant<16, 12, 1, 1>();
+        case 10: return eval_variant<16, 15, 1, 1, 1>();
+        case 11: return eval_variant<16, 8, 2, 1, 1>();
+        case 12: return eval_variant<16, 12, 1, 1, 1>();
+        case 13: return eval_variant<16, 16, 1, 1, 1>();
+        case 14: return eval_variant<16, 7, 2, 1, 1>();
         default: break;
         }
     }

@@ -171,7 +171,7 @@ __global__ void __launch_bounds__(kExhThreads) exh_kernel(ExhArgs a)
             const uint32_t k = s_qk[e];
             const uint64_t V = s_qv[e], bits = s_qb[e];
             const uint32_t OV = s_qo[e];
-            const double f = eq2(k, (int64_t)V, OV, T);
+            const double f = eq2(k, (int64_t)V, OV, T, a.m + 1, a.rcp);
             if (exh_better(f, bits, bf, bb)) {
                 bf = f;
                 bb = bits;

@@ -151,7 +151,7 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uin
     S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
     const uint64_t S1 = (uint64_t)ch.T + OV;
     const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
-    return eq2(k, V, OV, ch.T);
+    return eq2(k, V, OV, ch);
 }
 
 template <int WT>
@@ -194,7 +194,7 @@ __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* 
     const uint64_t S1 = (uint64_t)ch.T + OV;
     const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
     if (st) { st->k = k; st->V = V; st->S1 = S1; st->S2 = S2; st->OV = OV; }
-    return eq2(k, V, OV, ch.T);
+    return eq2(k, V, OV, ch);
 }
 
 // best-record order: (f desc, bitset asc; word W-1 most significant)
@@ -720,8 +720,8 @@ __device__ void leader_record(const GaArgs& a, uint32_t i, uint32_t g, uint32_t 
 // snapshot of an earlier record, list g%3).  R entries, the first kRecWin of
 // them staged in sm.rcw; rows and fitness are read from generation g.
 template <int WT>
-__device__ void leader_record_list(const GaArgs& a, uint32_t i, uint32_t g, uint32_t R, bool staged,
-                                   const Smem& sm)
+__device__ __forceinline__ BestRow<WT> rec_list_best(const GaArgs& a, uint32_t i, uint32_t g, uint32_t R, bool staged,
+                                                     const Smem& sm)
 {
     const uint32_t W = a.ch.W, L = g % 3u, cur = g & 1u;
     const uint64_t* popc = a.pop[cur] + (size_t)i * a.N * W;
@@ -739,11 +739,19 @@ __device__ void leader_record_list(const GaArgs& a, uint32_t i, uint32_t g, uint
         for (int w = 0; w < WT; ++w) o.r.w[w] = (w < (int)W) ? __ldcg(popc + (size_t)slot * W + w) : 0ull;
         if (better_row(o, v, W)) v = o;
     }
-    record_apply<WT>(a, i, g, v, R > 0, sm);
+    return v;
+}
+
+template <int WT>
+__device__ void leader_record_list(const GaArgs& a, uint32_t i, uint32_t g, uint32_t R, bool staged,
+                                   const Smem& sm)
+{
+    record_apply<WT>(a, i, g, rec_list_best<WT>(a, i, g, R, staged, sm), R > 0, sm);
 }
 
 // Copy the ranked elites (keys rk, indices rx into generation g) to slots
 // 0..E-1 of generation g+1 (R18) and publish the worst elite's key.
+template <int WT>
 __device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, const uint64_t* rk, const uint32_t* rx)
 {
     const uint32_t W = a.ch.W, N = a.N, E = a.E;
@@ -751,9 +759,11 @@ __device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, cons
     const uint64_t* popc = a.pop[cur] + (size_t)i * N * W;
     uint64_t* popn = a.pop[nxt] + (size_t)i * N * W;
     double* fitn = a.fit[nxt] + (size_t)i * a.Ns;
-    for (uint32_t j = threadIdx.x; j < E * W; j += blockDim.x) {
-        const uint32_t r = j / W, w = j % W;
-        popn[(size_t)r * W + w] = __ldcg(popc + (size_t)rx[r] * W + w);
+    // one row per thread per step: its W words are in flight together
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+        Row<WT> x;
+        row_load(x, popc + (size_t)rx[r] * W, W);
+        row_store(x, popn + (size_t)r * W, W);
     }
     for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(rk[r]);
     if (threadIdx.x == 0) a.tau[cur * a.I + i] = rk[E - 1];
@@ -761,10 +771,11 @@ __device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, cons
 
 // Leader, general path: the radix select already gathered the E best of
 // generation g; sort them and place them.
+template <int WT>
 __device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm)
 {
     leader_sort_selected(a, i, a.E, false, sm);
-    leader_copy_elites(a, i, g, sm.skey, sm.sidx);
+    leader_copy_elites<WT>(a, i, g, sm.skey, sm.sidx);
     __syncthreads();
 }
 
@@ -823,15 +834,33 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
         __syncthreads();
         C0 = sm.misc[3];
         if (C0 <= kCandCap) {
-            // gather every region into skey/sidx: warp w takes regions w, w+16, ...
-            const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+            // gather every region into skey/sidx.  Entry e of the concatenation lives in
+            // region c = max{c : cnt[c] <= e}; each thread issues all of its loads (one
+            // L2 round trip) before any shared-memory store.
             const uint64_t* ck = a.cand_key[Lc] + (size_t)i * cpi * a.creg;
             const uint32_t* cx = a.cand_idx[Lc] + (size_t)i * cpi * a.creg;
-            for (uint32_t c = warp; c < cpi; c += nwarps) {
-                const uint32_t o = cnt[c], nc = cnt[c + 1] - o;
-                for (uint32_t j = lane; j < nc; j += 32) {
-                    sm.skey[o + j] = __ldcg(ck + (size_t)c * a.creg + j);
-                    sm.sidx[o + j] = __ldcg(cx + (size_t)c * a.creg + j);
+            constexpr uint32_t kG = (kCandCap + kBlock - 1) / kBlock;
+            for (uint32_t e0 = 0; e0 < C0; e0 += kG * blockDim.x) {
+                uint64_t kk[kG];
+                uint32_t xx[kG];
+#pragma unroll
+                for (uint32_t u = 0; u < kG; ++u) {
+                    const uint32_t e = e0 + u * blockDim.x + threadIdx.x;
+                    if (e < C0) {
+                        uint32_t lo = 0, hi = cpi - 1;
+                        while (lo < hi) {
+                            const uint32_t mid = (lo + hi + 1) >> 1;
+                            if (cnt[mid] <= e) lo = mid; else hi = mid - 1;
+                        }
+                        const size_t src = (size_t)lo * a.creg + (e - cnt[lo]);
+                        kk[u] = __ldcg(ck + src);
+                        xx[u] = __ldcg(cx + src);
+                    }
+                }
+#pragma unroll
+                for (uint32_t u = 0; u < kG; ++u) {
+                    const uint32_t e = e0 + u * blockDim.x + threadIdx.x;
+                    if (e < C0) { sm.skey[e] = kk[u]; sm.sidx[e] = xx[u]; }
                 }
             }
         }
@@ -894,7 +923,7 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
         if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = sm.sidx[j]; }
     }
     __syncthreads();
-    leader_copy_elites(a, i, g, sm.okey, sm.oidx);
+    leader_copy_elites<WT>(a, i, g, sm.okey, sm.oidx);
     if (threadIdx.x == 0 && i == 0) a.ctl->n_fast = ++sm.misc[8];
     trace_mark(a, g, 3);
 }
@@ -1258,7 +1287,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             if (is_leader) {
                 // the record of generation g_begin was taken by INIT or at the end of
                 // the previous segment (and by the migrant import)
-                leader_general(a, blockIdx.x, g, sm);
+                leader_general<WT>(a, blockIdx.x, g, sm);
                 if (threadIdx.x == 0) {
                     a.rc_cnt[((g + 2u) % 3u) * I + blockIdx.x] = 0;
                     if (blockIdx.x == 0) a.ctl->n_general = ++sm.misc[9];
@@ -1322,7 +1351,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             // a candidate list overflowed: exact top-E of generation g (still intact)
             general_select(a, a.fit[cur], E, false, sm, grid);
             if (is_leader) {
-                leader_general(a, blockIdx.x, g, sm);
+                leader_general<WT>(a, blockIdx.x, g, sm);
                 if (threadIdx.x == 0 && blockIdx.x == 0) a.ctl->n_general = ++sm.misc[9];
             }
             grid.sync();

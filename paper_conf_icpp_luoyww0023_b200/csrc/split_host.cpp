@@ -228,6 +228,39 @@ static int dalloc(split_ga_t* h, T** out, size_t count)
     return SPLIT_OK;
 }
 
+// Device arena: create() plans every buffer, then makes ONE cudaMalloc and one
+// stream-ordered memset (dozens of separate cudaMalloc/cudaMemset calls cost
+// milliseconds per handle, which the end-to-end path pays on every create).
+struct DevPlan {
+    std::vector<std::pair<void**, size_t>> req;
+    template <class T>
+    void add(T** out, size_t count)
+    {
+        *out = nullptr;
+        req.push_back({(void**)out, std::max<size_t>(count * sizeof(T), 16)});
+    }
+};
+
+static int commit_plan(split_ga_t* h, DevPlan& pl)
+{
+    size_t total = 0;
+    for (auto& r : pl.req) total = ((total + 255) & ~(size_t)255) + r.second;
+    void* base = nullptr;
+    cudaError_t e = cudaMalloc(&base, total);
+    if (e != cudaSuccess) return fail(SPLIT_E_NOMEM, "cudaMalloc(%zu): %s", total, cudaGetErrorString(e));
+    h->allocs.push_back(base);
+    size_t off = 0;
+    for (auto& r : pl.req) {
+        off = (off + 255) & ~(size_t)255;
+        *r.first = (uint8_t*)base + off;
+        off += r.second;
+    }
+    e = cudaMemsetAsync(base, 0, total, h->stream);
+    if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "cudaMemsetAsync: %s", cudaGetErrorString(e));
+    pl.req.clear();
+    return SPLIT_OK;
+}
+
 static uint64_t bern_thr(double p)
 {
     if (!(p > 0.0)) return 0;
@@ -325,16 +358,6 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     }
     words[n] = (uint32_t)acc;
     for (uint32_t i = 0; i + 1 < n; ++i) words[p_words + i] = (uint32_t)ovh[i];
-    uint32_t* d_chain = nullptr;
-    TRY(dalloc(h, &d_chain, words.size()));
-    {
-        cudaError_t e = cudaMemcpy(d_chain, words.data(), words.size() * 4, cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) {
-            free_all(h);
-            delete h;
-            return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
-        }
-    }
     // interleaved {P[p+1], ovh[p]} table for the eval kernel's walk
     const uint32_t po_n = ((n - 1) + 1) & ~1u;                  // entries, even -> 16-byte multiple
     std::vector<uint32_t> po(2 * (size_t)po_n, 0);
@@ -342,22 +365,24 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
         po[2 * q] = words[q + 1];
         po[2 * q + 1] = (uint32_t)ovh[q];
     }
+    DevPlan plan;
+    uint32_t* d_chain = nullptr;
     uint32_t* d_po = nullptr;
-    TRY(dalloc(h, &d_po, po.size()));
-    {
-        cudaError_t e = cudaMemcpy(d_po, po.data(), po.size() * 4, cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) {
-            free_all(h);
-            delete h;
-            return fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e));
-        }
+    plan.add(&d_chain, words.size());
+    plan.add(&d_po, po.size());
+    // Eq. 2 reciprocals (ChainDev::rcp): IEEE divisions, i.e. correctly rounded
+    std::vector<double> rcp(2 * (size_t)n + 2, 0.0);
+    rcp[0] = 1.0 / (double)acc;
+    for (uint32_t k = 1; k <= n; ++k) {
+        rcp[k] = 1.0 / (double)k;
+        rcp[n + 1 + k] = 1.0 / ((double)k * (double)acc);   // k T < 2^53: exact product
     }
+    double* d_rcp = nullptr;
+    plan.add(&d_rcp, rcp.size());
     h->hwords = words;
     h->p_words = p_words;
     ChainDev& ch = h->ch;
-    ch.po = (const uint2*)d_po;
     ch.po_bytes = (uint32_t)(po.size() * 4);
-    ch.words = d_chain;
     ch.n = n;
     ch.W = h->W;
     ch.p_words = p_words;
@@ -416,8 +441,8 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     h->cpi = a.cpi;
     const size_t IN = (size_t)a.I * a.N, INs = (size_t)a.I * a.Ns;
     for (int b = 0; b < 2; ++b) {
-        TRY(dalloc(h, &a.pop[b], IN * h->W));
-        TRY(dalloc(h, &a.fit[b], INs));
+        plan.add(&a.pop[b], IN * h->W);
+        plan.add(&a.fit[b], INs);
     }
     {
         // candidate regions: worker CTA c of an island produces at most 32 children per
@@ -426,37 +451,49 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
         a.creg = 32u * ((chunks + a.cpi - 1u) / a.cpi) + 32u;
     }
     for (int b = 0; b < 3; ++b) {
-        TRY(dalloc(h, &a.cand_key[b], (size_t)a.I * a.cpi * a.creg));
-        TRY(dalloc(h, &a.cand_idx[b], (size_t)a.I * a.cpi * a.creg));
+        plan.add(&a.cand_key[b], (size_t)a.I * a.cpi * a.creg);
+        plan.add(&a.cand_idx[b], (size_t)a.I * a.cpi * a.creg);
     }
-    TRY(dalloc(h, &a.cand_cnt, 3 * (size_t)a.I * a.cpi_pad));
-    TRY(dalloc(h, &a.rc_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4));
-    for (int b = 0; b < 3; ++b) TRY(dalloc(h, &a.rc_idx[b], INs));
-    TRY(dalloc(h, &a.snap_f, 2 * (size_t)a.I));
-    TRY(dalloc(h, &a.snap_bits, 2 * (size_t)a.I * h->W));
-    TRY(dalloc(h, &a.sel_key, (size_t)a.I * kMaxElite));
-    TRY(dalloc(h, &a.sel_idx, (size_t)a.I * kMaxElite));
-    TRY(dalloc(h, &a.sel_cnt, a.I));
-    TRY(dalloc(h, &a.tau, 2 * (size_t)a.I));
-    TRY(dalloc(h, &a.ghist, 3 * (size_t)a.I * 256));
-    TRY(dalloc(h, &a.part_f, 2 * (size_t)a.I * a.cpi_pad));
-    TRY(dalloc(h, &a.part_idx, 2 * (size_t)a.I * a.cpi_pad));
-    TRY(dalloc(h, &a.part_bits, 2 * (size_t)a.I * a.cpi_pad * h->W));
-    TRY(dalloc(h, &a.rec_f, a.I));
-    TRY(dalloc(h, &a.rec_bits, (size_t)a.I * h->W));
-    TRY(dalloc(h, &a.rec_gen, a.I));
-    TRY(dalloc(h, &a.rec_valid, a.I));
-    TRY(dalloc(h, &a.mig_bits, (size_t)a.I_total * std::max<uint32_t>(a.K, 1) * h->W));
-    TRY(dalloc(h, &a.mig_f, (size_t)a.I_total * std::max<uint32_t>(a.K, 1)));
-    TRY(dalloc(h, &a.ctl, 1));
-    TRY(dalloc(h, &a.gbar, 4));
-    TRY(dalloc(h, &h->d_stats, 8));
-    TRY(dalloc(h, &h->d_statf, 1));
-    TRY(dalloc(h, &h->d_bits1, h->W));
-    TRY(dalloc(h, &h->d_recpack, (size_t)a.I_total * (h->W + 2)));
+    plan.add(&a.cand_cnt, 3 * (size_t)a.I * a.cpi_pad);
+    plan.add(&a.rc_cnt, ((3 * (size_t)a.I + 3) & ~(size_t)3) + 4);
+    for (int b = 0; b < 3; ++b) plan.add(&a.rc_idx[b], INs);
+    plan.add(&a.snap_f, 2 * (size_t)a.I);
+    plan.add(&a.snap_bits, 2 * (size_t)a.I * h->W);
+    plan.add(&a.sel_key, (size_t)a.I * kMaxElite);
+    plan.add(&a.sel_idx, (size_t)a.I * kMaxElite);
+    plan.add(&a.sel_cnt, a.I);
+    plan.add(&a.tau, 2 * (size_t)a.I);
+    plan.add(&a.ghist, 3 * (size_t)a.I * 256);
+    plan.add(&a.part_f, 2 * (size_t)a.I * a.cpi_pad);
+    plan.add(&a.part_idx, 2 * (size_t)a.I * a.cpi_pad);
+    plan.add(&a.part_bits, 2 * (size_t)a.I * a.cpi_pad * h->W);
+    plan.add(&a.rec_f, a.I);
+    plan.add(&a.rec_bits, (size_t)a.I * h->W);
+    plan.add(&a.rec_gen, a.I);
+    plan.add(&a.rec_valid, a.I);
+    plan.add(&a.mig_bits, (size_t)a.I_total * std::max<uint32_t>(a.K, 1) * h->W);
+    plan.add(&a.mig_f, (size_t)a.I_total * std::max<uint32_t>(a.K, 1));
+    plan.add(&a.ctl, 1);
+    plan.add(&a.gbar, 4);
+    plan.add(&h->d_stats, 8);
+    plan.add(&h->d_statf, 1);
+    plan.add(&h->d_bits1, h->W);
+    plan.add(&h->d_recpack, (size_t)a.I_total * (h->W + 2));
     if (getenv("SPLIT_TRACE")) {
         h->trace_gens = 64;
-        TRY(dalloc(h, &h->d_trace, (size_t)h->trace_gens * 16));
+        plan.add(&h->d_trace, (size_t)h->trace_gens * 16);
+    }
+    TRY(commit_plan(h, plan));
+    ch.po = (const uint2*)d_po;
+    ch.words = d_chain;
+    ch.rcp = d_rcp;
+    a.ch = ch;
+    {
+        cudaError_t e = cudaMemcpyAsync(d_chain, words.data(), words.size() * 4, cudaMemcpyHostToDevice, h->stream);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(d_po, po.data(), po.size() * 4, cudaMemcpyHostToDevice, h->stream);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(d_rcp, rcp.data(), rcp.size() * 8, cudaMemcpyHostToDevice, h->stream);
+        // (pageable sources: the calls return once the host data has been staged)
+        if (e != cudaSuccess) TRY(fail(SPLIT_E_CUDA, "chain upload: %s", cudaGetErrorString(e)));
     }
     for (int i = 0; i < 4; ++i) {
         cudaError_t e = cudaEventCreate(&h->ev[i]);
@@ -877,6 +914,7 @@ extern "C" int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* 
     a.m = m;
     a.c = c;
     a.T = (uint32_t)h->T;
+    a.rcp = h->ch.rcp;
     a.k_min = h->p.k_min;
     a.k_max = h->p.k_max;
     a.outer_total = (uint64_t)1 << (m - c);

@@ -38,6 +38,9 @@ struct ChainDev {
     uint64_t last_mask;         // valid bits of word W-1
     const uint2* po;            // device: po[p] = {P[p+1], ovh[p]}, p in [0, n-2] (padded)
     uint32_t po_bytes;          // multiple of 16
+    // correctly rounded reciprocals for Eq. 2's divisions (split_device.cuh div_rcp_rn):
+    // rcp[0] = RN(1/T), rcp[k] = RN(1/k) and rcp[n + 1 + k] = RN(1/(k T)) for k in [1, n]
+    const double* rcp;          // device, 2n + 2 entries
 };
 
 // All device pointers and scalars the GA kernel needs (passed by value).
@@ -96,6 +99,7 @@ struct ExhArgs {
     void* tab;             // [(m-c+1) << c] ExhEntry
     uint32_t m, c;         // cut positions n-1, low positions
     uint32_t T, k_min, k_max;
+    const double* rcp;     // ChainDev::rcp of the chain (n = m + 1)
     uint64_t outer_total;  // 2^(m-c) high-part states
     uint64_t per_thread;   // high-part states per thread
     void* res;             // [grid] per-CTA best (MODE_EXH_BEST)
