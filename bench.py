@@ -36,6 +36,9 @@ C2 = dict(chain="resnet50_175", pop_size=65536, n_elite=1024, tournament_size=4,
 MIGRATION_INTERVAL, N_MIGRANTS = 10, 64
 C5_EVAL_N = 1 << 24           # split_eval_batch sub-measurement (C5: n = 1024, 2.3 GB of bitsets > L2)
 EXACT_N = 33                  # f1 sub-measurement: split_exhaustive over 2^32 splits
+QOS_REPLICAS = 65536          # f2 sub-measurement
+GA_BIG = dict(chain="bert_base", pop_size=1 << 22, n_elite=1024, tournament_size=4, p_crossover=0.9,
+              p_mutation=0.2, k_min=2, k_max=32, generations=50)   # C4-shaped island of 4M: HBM regime
 CPU_SAMPLE_GENERATIONS = 100  # oracle cpu_baseline: about 10 s of one core
 REF_STEP_GENERATIONS = 10     # --impl reference: oracle generations per step
 
@@ -201,6 +204,8 @@ def main():
     ap.add_argument("--no-eval", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-exact", action="store_true")
+    ap.add_argument("--no-ga-big", action="store_true")
+    ap.add_argument("--no-qos", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
@@ -300,12 +305,21 @@ def main():
     if not args.no_e2e:
         e2e_steps = max(3, min(args.steps, 10))
         e_evals = 0
+        with S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl) as he:   # warm-up
+            he.run(G, 4999)
         barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
+        e_wall = []
         for i in range(e2e_steps):
-            with S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl) as he:
-                e_evals += he.run(G, 5000 + i)["evaluations"]
+            ti = time.perf_counter()
+            he = S.SplitGA(lat, ovh, device=local, stream=stream, comm=comm, **gkw, **isl)
+            tc = time.perf_counter()
+            e_evals += he.run(G, 5000 + i)["evaluations"]
+            tr = time.perf_counter()
+            he.close()
+            td = time.perf_counter()
+            e_wall.append([round((tc - ti) * 1e3, 3), round((tr - tc) * 1e3, 3), round((td - tr) * 1e3, 3)])
         torch.cuda.synchronize()
         barrier()
         et_s, ee_all, _ = D.reduce_max_sum(time.perf_counter() - t0, float(e_evals), device=dev)
@@ -313,7 +327,7 @@ def main():
         h2d = 4 * (((n + 1 + 3) & ~3) + ((n - 1 + 3) & ~3)) + 8   # staged chain words + best bits
         d2h = 48 + world * (W + 2) * 8 + 5 * 8 + 8                # control block, island records, best stats
         out["e2e"] = {"value": ee_all / et_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
-                      "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+                      "d2h_bytes_per_step": d2h, "steps": e2e_steps, "wall_ms_create_run_destroy": e_wall,
                       "note": "split_ga_create(host latencies) + split_ga_run + best to host + destroy, wall clock"}
 
     # split_eval_batch at C5 (HBM-bound; the north-star's >= 60 % target)
@@ -347,6 +361,75 @@ def main():
                          "algorithmic_bytes_per_candidate": bpc}}
         h5.close()
         del bits, fout
+
+    # the same GA kernel on one C4-shaped island of 4M individuals (BERT-base chain, W = 7):
+    # 235 MB of population per generation buffer, far above L2 -> the HBM regime
+    if not args.no_ga_big:
+        latb, ovhb = wl.chain(GA_BIG["chain"])
+        bkw = {k: GA_BIG[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation",
+                                      "k_min", "k_max")}
+        with S.SplitGA(latb, ovhb, device=local, stream=stream, **bkw) as hb:
+            Gb = GA_BIG["generations"]
+            hb.run(Gb, 77)
+            bm, bev, bloop = [], 0, []
+            for i in range(3):
+                flush.fill_(i)
+                b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                b0.record(stream)
+                rb = hb.run(Gb, 100 + i)
+                b1.record(stream)
+                torch.cuda.synchronize()
+                bm.append(b0.elapsed_time(b1))
+                bev += rb["evaluations"]
+                bloop.append(hb.last_run_stats()["ms_loop"])
+            Wb = hb.W
+        bms = sum(bm) / len(bm)
+        gbytes = ga_bytes_per_generation(GA_BIG["pop_size"], GA_BIG["n_elite"], Wb, GA_BIG["tournament_size"])
+        bl = sum(bloop) / len(bloop)
+        bgbs = gbytes * Gb / (bl / 1000.0) / 1e9
+        out["ga_hbm_regime"] = {
+            "workload": f"C4-shaped island on one GPU: bert_base chain (n=400, W={Wb}), pop={GA_BIG['pop_size']}, "
+                        f"E=1024, s=4, {Gb} generations per step",
+            "evals_per_s": bev / (sum(bm) / 1000.0), "ms_per_step": bms,
+            "gens_per_s": Gb / (bms / 1000.0),
+            "roofline": {"bound": "hbm", "kernel": "ga_kernel (RUN segment)", "achieved": bgbs,
+                         "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": bgbs / peaks["hbm_gbs"],
+                         "peak_src": peaks["src"], "algorithmic_bytes_per_generation": gbytes,
+                         "launch_ms_avg": bl}}
+
+    # f2 QoS simulator: Table 2's heaviest scenario (lambda = 110 ms, 1000 requests) over the
+    # paper-five chains split into 4 blocks by the GA, Algorithm 1 vs FIFO, 65,536 replicas
+    if not args.no_qos:
+        qb = []
+        for name in ("yolov2", "googlenet", "resnet50_122", "vgg19", "gpt2"):
+            lq, oq = wl.chain(name)
+            with S.SplitGA(lq, oq, pop_size=4096, n_elite=64, k_min=4, k_max=4, device=local, stream=stream) as hq:
+                rq = hq.run(50, 1)
+            qb.append(S.block_times(lq, oq, rq["bits"]))
+        arr, typ = wl.qos_requests(QOS_REPLICAS, 1000, 110_000_000, len(qb), seed=2023)
+        da, dt = torch.from_numpy(arr).to(dev), torch.from_numpy(typ).to(dev)
+        alphas = [1000 * a for a in range(2, 21)]
+        qout = {}
+        for pol, pname in ((1, "algorithm1"), (0, "fifo")):
+            S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream)
+            torch.cuda.synchronize()
+            q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            q0.record(stream)
+            te, viol, rr = S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream)
+            q1.record(stream)
+            torch.cuda.synchronize()
+            qms = q0.elapsed_time(q1)
+            v = viol.cpu().numpy().view(np.uint32).astype(np.float64).sum(axis=0) / (QOS_REPLICAS * 1000)
+            r = rr.cpu().numpy()
+            mean = r[:, 0].sum() / (QOS_REPLICAS * 1000)
+            sd = float(np.sqrt(max(r[:, 1].sum() / (QOS_REPLICAS * 1000) - mean * mean, 0.0)))
+            qout[pname] = {"requests_per_s": QOS_REPLICAS * 1000 / (qms / 1000.0), "ms": qms,
+                           "violation_rate": {f"alpha={a // 1000}": float(x) for a, x in zip(alphas, v)},
+                           "rr_mean": float(mean), "rr_std": sd}
+        out["qos_sim"] = {"workload": f"f2: {QOS_REPLICAS} replicas x 1000 Poisson requests (lambda = 110 ms), "
+                                      "paper-five chains in 4 GA-chosen blocks each",
+                          "blocks_ms": [[round(b / 1e6, 3) for b in bl] for bl in qb], **qout}
+        del da, dt
 
     # f1 exact solver: exhaustive enumeration of all 2^32 splits of a 33-op chain
     if not args.no_exact:

@@ -149,6 +149,31 @@ typedef struct {
 } split_queue_state;
 int split_preempt_decide(const split_queue_state* q, uint32_t* insert_pos);
 
+/* f2 — QoS simulator (R20).  Batched Monte-Carlo
+ * of one edge executor serving requests of n_types split models: requests are
+ * preempted only between blocks (§3.4, P@24400-26700), the queue order is
+ * decided at each arrival by Algorithm 1 (policy 1, the closed form of
+ * split_preempt_decide) or FIFO (policy 0), the latency target is alpha*Ext
+ * (fn. 3, P@29746-29870) and a request violates it when t_ete/Ext > alpha
+ * (Eq. 3, §5.2).  One replica per GPU thread; everything is integer ns.
+ *   blocks_ns    host, sum(n_blocks) entries: model m's blocks in order, each in
+ *                [1, 2^32); Ext(m) = sum of its blocks < 2^32
+ *   n_blocks     host, n_types entries (1..65535); n_types in [1, 65535]
+ *   arrival_ns   device int64 [n_rep][n_req], non-decreasing per replica, >= 0
+ *   type_id      device uint32 [n_rep][n_req], < n_types
+ *   alpha_milli  host, n_alpha (<= 32) thresholds alpha*1000 (> 0)
+ *   t_ete_out    device int64 [n_rep][n_req]: end-to-end latency per request
+ *   viol_out     device uint32 [n_rep][n_alpha]: #{i : 1000 t_ete > alpha_milli Ext}
+ *   rr_out       device double [n_rep][2]: sum of t_ete/Ext and of its square,
+ *                added in request order
+ * Synchronous.  SPLIT_E_INVAL on bad host arguments; SPLIT_E_RANGE when a
+ * replica has unordered arrivals / a bad type id or more than 32 pending
+ * requests (an overloaded system: its results are then undefined). */
+int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
+                       const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep, uint32_t n_req,
+                       const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,
+                       uint32_t* viol_out, double* rr_out, int device, void* stream);
+
 /* Island communicator over NCCL (the libnccl.so.2 already loaded in the
  * process, e.g. by torch).  Rank r of `world` runs islands_per_device islands
  * starting at island_id = r*islands_per_device.  unique_id: 128 bytes from

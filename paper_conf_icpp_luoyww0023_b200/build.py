@@ -11,7 +11,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB_DIR = os.path.join(PKG, "lib")
 LIB = os.path.join(LIB_DIR, "libsplit_ga.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("split_eval.cu", "split_ga.cu", "split_exact.cu", "split_host.cpp")]
+SOURCES = [os.path.join(CSRC, f) for f in ("split_eval.cu", "split_ga.cu", "split_exact.cu", "split_qos.cu", "split_host.cpp")]
 HEADERS = [os.path.join(CSRC, "split_internal.h"), os.path.join(CSRC, "split_device.cuh"),
            os.path.join(ROOT, "include", "split_ga.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

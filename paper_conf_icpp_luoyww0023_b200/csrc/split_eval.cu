@@ -371,6 +371,11 @@ static EvalVariant eval_pick(uint32_t W)
         case 12: return eval_variant<16, 12, 1, 1, 1>();
         case 13: return eval_variant<16, 16, 1, 1, 1>();
         case 14: return eval_variant<16, 7, 2, 1, 1>();
+        case 15: return eval_variant<16, 11, 1, 1>();
+        case 16: return eval_variant<16, 9, 1, 1>();
+        case 17: return eval_variant<16, 7, 1, 1>();
+        case 18: return eval_variant<16, 6, 1, 1>();
+        case 19: return eval_variant<16, 5, 1, 1>();
         default: break;
         }
     }

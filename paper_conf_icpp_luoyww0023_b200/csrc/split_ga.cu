@@ -789,7 +789,7 @@ __device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Sm
 template <int WT>
 __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm, uint32_t& mph)
 {
-    const uint32_t W = a.ch.W, Ns = a.Ns, E = a.E, I = a.I, cpi = a.cpi, cpp = a.cpi_pad;
+    const uint32_t Ns = a.Ns, E = a.E, I = a.I, cpi = a.cpi, cpp = a.cpi_pad;
     const uint32_t cur = g & 1u, Lc = g % 3u, Lr = (g + 2u) % 3u;
     trace_mark(a, g, 0);
     if (threadIdx.x == 0) {

@@ -1011,3 +1011,76 @@ extern "C" int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out)
     h->stats.ms_loop = h->stats.ms_total;
     return SPLIT_OK;
 }
+
+// ------------------------------------------------------------------------
+// f2: QoS simulator (split_qos.cu)
+// ------------------------------------------------------------------------
+extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
+                                  const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep, uint32_t n_req,
+                                  const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,
+                                  uint32_t* viol_out, double* rr_out, int device, void* stream)
+{
+    if (!blocks_ns || !n_blocks || n_types == 0 || n_types > 65535)
+        return fail(SPLIT_E_INVAL, "split_qos_simulate: need 1..65535 model types with their blocks");
+    if (policy > 1) return fail(SPLIT_E_INVAL, "split_qos_simulate: policy must be 0 (FIFO) or 1 (Algorithm 1)");
+    if (n_alpha > kQosMaxAlpha || (n_alpha && !alpha_milli))
+        return fail(SPLIT_E_INVAL, "split_qos_simulate: at most %u alpha thresholds", kQosMaxAlpha);
+    if (n_rep == 0 || n_req == 0) return SPLIT_OK;
+    if (!arrival_ns || !type_id || !t_ete_out || !rr_out || (n_alpha && !viol_out))
+        return fail(SPLIT_E_INVAL, "split_qos_simulate: NULL device buffer");
+    std::vector<uint32_t> off(n_types + 1, 0), ext(n_types, 0), blk;
+    for (uint32_t m = 0; m < n_types; ++m) {
+        if (n_blocks[m] == 0 || n_blocks[m] > 65535)
+            return fail(SPLIT_E_INVAL, "split_qos_simulate: model %u has %u blocks (need 1..65535)", m, n_blocks[m]);
+        uint64_t e = 0;
+        for (uint32_t j = 0; j < n_blocks[m]; ++j) {
+            const int64_t b = blocks_ns[off[m] + j];
+            if (b < 1 || b >= ((int64_t)1 << 32)) return fail(SPLIT_E_RANGE, "split_qos_simulate: block time out of [1, 2^32)");
+            e += (uint64_t)b;
+            blk.push_back((uint32_t)b);
+        }
+        if (e >= ((uint64_t)1 << 32)) return fail(SPLIT_E_RANGE, "split_qos_simulate: Ext(model %u) >= 2^32 ns", m);
+        ext[m] = (uint32_t)e;
+        off[m + 1] = off[m] + n_blocks[m];
+    }
+    for (uint32_t j = 0; j < n_alpha; ++j)
+        if (alpha_milli[j] == 0) return fail(SPLIT_E_INVAL, "split_qos_simulate: alpha must be > 0");
+    CU(cudaSetDevice(device));
+    cudaStream_t st = (cudaStream_t)stream;
+    std::vector<uint32_t> tab;
+    tab.insert(tab.end(), off.begin(), off.end());
+    tab.insert(tab.end(), ext.begin(), ext.end());
+    tab.insert(tab.end(), alpha_milli, alpha_milli + n_alpha);
+    tab.insert(tab.end(), blk.begin(), blk.end());
+    tab.push_back(0);                                   // error flag
+    QosArgs a;
+    memset(&a, 0, sizeof(a));
+    a.n_types = n_types;
+    a.n_blocks_total = (uint32_t)blk.size();
+    a.n_alpha = n_alpha;
+    a.policy = policy;
+    a.n_rep = n_rep;
+    a.n_req = n_req;
+    a.arrival = arrival_ns;
+    a.type = type_id;
+    a.t_ete = t_ete_out;
+    a.viol = viol_out;
+    a.rr = rr_out;
+    if (qos_smem_bytes(a) > 227 * 1024) return fail(SPLIT_E_INVAL, "split_qos_simulate: model tables too large");
+    DevScratch sc;
+    uint32_t* d_tab;
+    RC(sc.alloc(&d_tab, tab.size()));
+    CU(cudaMemcpyAsync(d_tab, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice, st));
+    a.blk_off = d_tab;
+    a.ext = d_tab + n_types + 1;
+    a.alpha_milli = a.ext + n_types;
+    a.blk_ns = a.alpha_milli + n_alpha;
+    a.err = d_tab + tab.size() - 1;
+    CU(launch_qos(a, st));
+    uint32_t err = 0;
+    CU(cudaMemcpyAsync(&err, a.err, 4, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    if (err == 1) return fail(SPLIT_E_RANGE, "split_qos_simulate: arrivals not non-decreasing / negative, or type id >= n_types");
+    if (err == 2) return fail(SPLIT_E_RANGE, "split_qos_simulate: more than %u pending requests (overloaded)", kQosQueue);
+    return SPLIT_OK;
+}

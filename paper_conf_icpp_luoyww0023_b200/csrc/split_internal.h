@@ -109,6 +109,28 @@ struct ExhArgs {
 };
 size_t exh_smem_bytes(const ExhArgs& a);
 int exh_blocks_per_sm(const ExhArgs& a);
+// f2 QoS simulator (split_qos.cu)
+constexpr uint32_t kQosThreads = 128;   // replicas per CTA (one per thread)
+constexpr uint32_t kQosQueue = 32;      // pending requests a replica may hold
+constexpr uint32_t kQosMaxAlpha = 32;
+struct QosArgs {
+    uint32_t n_types, n_blocks_total, n_alpha, policy;
+    const uint32_t* blk_off;       // [n_types + 1] prefix of blocks per type
+    const uint32_t* blk_ns;        // [n_blocks_total]
+    const uint32_t* ext;           // [n_types] Ext = sum of the type's blocks
+    const uint32_t* alpha_milli;   // [n_alpha]
+    uint64_t n_rep;
+    uint32_t n_req;
+    const int64_t* arrival;        // [n_rep][n_req]
+    const uint32_t* type;          // [n_rep][n_req]
+    int64_t* t_ete;                // [n_rep][n_req]
+    uint32_t* viol;                // [n_rep][n_alpha]
+    double* rr;                    // [n_rep][2]
+    uint32_t* err;                 // 0 ok, 1 bad arrival/type, 2 queue overflow
+};
+size_t qos_smem_bytes(const QosArgs& a);
+cudaError_t launch_qos(const QosArgs& a, cudaStream_t st);
+
 cudaError_t launch_exh_table(const ExhArgs& a, cudaStream_t st);
 cudaError_t launch_exh(const ExhArgs& a, int mode, uint32_t grid, cudaStream_t st);
 cudaError_t launch_exh_reduce(const void* res, uint32_t n, void* out, cudaStream_t st);

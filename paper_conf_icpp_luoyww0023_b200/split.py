@@ -76,6 +76,9 @@ def _load():
         "split_ga_run": (C.c_int, [C.c_void_p, C.c_uint32, C.c_uint64, P(split_best_t)]),
         "split_ga_population": (C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
         "split_preempt_decide": (C.c_int, [P(split_queue_state), P(C.c_uint32)]),
+        "split_qos_simulate": (C.c_int, [P(C.c_int64), P(C.c_uint32), C.c_uint32, C.c_uint32, P(C.c_uint32),
+                                         C.c_uint32, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p, C.c_void_p,
+                                         C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),
         "split_comm_unique_id": (C.c_int, [C.c_void_p]),
         "split_comm_init": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, P(C.c_void_p)]),
         "split_comm_destroy": (None, [C.c_void_p]),
@@ -100,7 +103,7 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_eval_batch_host", "split_ga_run", "split_ga_population", "split_preempt_decide",
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
-            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2")
+            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate")
 
 
 def lib():
@@ -137,6 +140,44 @@ def split_preempt_decide(now_ns: int, alpha: float, queue, incoming) -> int:
     pos = C.c_uint32(0)
     _check(_lib.split_preempt_decide(C.byref(q), C.byref(pos)), "split_preempt_decide")
     return int(pos.value)
+
+
+def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int = 0, stream=None):
+    """f2 QoS simulator (include/split_ga.h).  blocks: per model type, its block
+    times (ns); arrival: device int64 tensor [n_rep, n_req]; type_id: device int32
+    tensor of the same shape.  Returns device tensors (t_ete [n_rep, n_req] int64,
+    violations [n_rep, n_alpha] int32 (uint32 bits), rr [n_rep, 2] f64)."""
+    import torch
+    n_rep, n_req = arrival.shape
+    flat = np.ascontiguousarray(np.concatenate([np.asarray(b, dtype=np.int64) for b in blocks]))
+    nb = np.ascontiguousarray(np.array([len(b) for b in blocks], dtype=np.uint32))
+    al = np.ascontiguousarray(np.asarray(alpha_milli, dtype=np.uint32))
+    dev = arrival.device
+    t_ete = torch.empty((n_rep, n_req), dtype=torch.int64, device=dev)
+    viol = torch.empty((n_rep, max(len(al), 1)), dtype=torch.int32, device=dev)
+    rr = torch.empty((n_rep, 2), dtype=torch.float64, device=dev)
+    assert arrival.dtype == torch.int64 and arrival.is_contiguous()
+    assert type_id.dtype == torch.int32 and type_id.is_contiguous() and type_id.shape == arrival.shape
+    _check(lib().split_qos_simulate(flat.ctypes.data_as(C.POINTER(C.c_int64)), nb.ctypes.data_as(C.POINTER(C.c_uint32)),
+                                    len(blocks), policy, al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep,
+                                    n_req, arrival.data_ptr(), type_id.data_ptr(), t_ete.data_ptr(), viol.data_ptr(),
+                                    rr.data_ptr(), device, _stream_handle(stream)), "split_qos_simulate")
+    return t_ete, viol, rr
+
+
+def block_times(latencies_ns, cut_overhead_ns, bits) -> list[int]:
+    """Block execution times (ns) of a split under the additive model (R2, R3):
+    the block after cut p pays ovh[p].  bits: the split's W words (host)."""
+    lat = np.asarray(latencies_ns, dtype=np.int64)
+    ovh = np.zeros(len(lat) - 1, dtype=np.int64) if cut_overhead_ns is None else np.asarray(cut_overhead_ns, np.int64)
+    out, cur = [], 0
+    for p in range(len(lat)):
+        cur += int(lat[p])
+        if p < len(lat) - 1 and (int(bits[p >> 6]) >> (p & 63)) & 1:
+            out.append(cur)
+            cur = int(ovh[p])
+    out.append(cur)
+    return out
 
 
 def split_comm_unique_id() -> bytes:

@@ -209,3 +209,27 @@ def uniform_k_population_fast(n_ops: int, n_cand: int, seed: int, k_lo: int = 2,
     bit = np.left_shift(np.uint64(1), (p & 63).astype(np.uint64))
     np.bitwise_or.at(out, (rows, p >> 6), bit)
     return out
+
+
+def qos_requests(n_rep: int, n_req: int, lam_ns: int, n_types: int, seed: int):
+    """Poisson request streams for the f2 simulator (§5.1, Table 2 P@31725-32980:
+    mean arrival interval lambda, here in ns): per replica, exponential
+    inter-arrival gaps rounded to integer ns (cumulative, starting at the first
+    gap) and a model type uniform in [0, n_types).  Returns (arrival int64
+    [n_rep, n_req], type int32 [n_rep, n_req])."""
+    rng = np.random.default_rng(seed)
+    gaps = np.rint(rng.exponential(float(lam_ns), size=(n_rep, n_req))).astype(np.int64)
+    arrival = np.cumsum(gaps, axis=1)
+    types = rng.integers(0, n_types, size=(n_rep, n_req), dtype=np.int32)
+    return arrival, types
+
+
+def random_blocks(n_types: int, seed: int, k_lo: int = 1, k_hi: int = 6, lo: int = 200_000, hi: int = 20_000_000):
+    """Random per-model block lists (ns) for simulator tests: k in [k_lo, k_hi]
+    blocks per model, each uniform in [lo, hi)."""
+    rng = np.random.default_rng(seed)
+    out = []
+    for _ in range(n_types):
+        k = int(rng.integers(k_lo, k_hi + 1))
+        out.append([int(x) for x in rng.integers(lo, hi, size=k)])
+    return out

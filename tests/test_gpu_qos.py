@@ -1,0 +1,105 @@
+"""GPU parity of the f2 QoS simulator (split_qos_simulate, R20)
+against oracle/qos.py (literal Algorithm 1 in exact rationals, or FIFO):
+end-to-end latency of every request, violation counts per alpha and both
+response-ratio sums, bit for bit.  Small cases compare every replica; the
+bench-sized case (Table 2's 1000 requests, lambda = 110 ms, 8192 replicas)
+compares sampled replicas plus properties that hold at any size."""
+import numpy as np
+import pytest
+
+from oracle import qos as Q
+from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ALPHAS = [1000 * a for a in range(2, 21)] + [1500]
+
+
+@pytest.fixture(scope="module")
+def S():
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA not available on a GPU test run")
+    from paper_conf_icpp_luoyww0023_b200 import split
+    return split
+
+
+def _run(S, blocks, arr, ty, policy, alphas=ALPHAS):
+    a = torch.from_numpy(arr).cuda()
+    t = torch.from_numpy(ty).cuda()
+    te, viol, rr = S.split_qos_simulate(blocks, a, t, alphas, policy)
+    torch.cuda.synchronize()
+    return te.cpu().numpy(), viol.cpu().numpy().view(np.uint32), rr.cpu().numpy()
+
+
+def _check_replica(blocks, arr, ty, policy, te, viol, rr, alphas=ALPHAS):
+    a = [int(x) for x in arr]
+    t = [int(x) for x in ty]
+    want = Q.simulate(blocks, a, t, policy)
+    assert [int(x) for x in te] == want
+    v, rs, rq = Q.stats(blocks, t, want, alphas)
+    assert [int(x) for x in viol[:len(alphas)]] == v
+    assert rr[0] == rs and rr[1] == rq          # bit-identical sums
+
+
+@pytest.mark.parametrize("policy", [Q.FIFO, Q.ALG1])
+@pytest.mark.parametrize("seed", [1, 42, 20230807])
+def test_small_cases_all_replicas(S, policy, seed):
+    blocks = wl.random_blocks(5, seed=seed, k_hi=6, lo=300_000, hi=9_000_000)
+    arr, ty = wl.qos_requests(37, 150, 40_000_000, 5, seed=seed)   # ragged: 37 replicas (one partial CTA)
+    te, viol, rr = _run(S, blocks, arr, ty, policy)
+    for r in range(arr.shape[0]):
+        _check_replica(blocks, arr[r], ty[r], policy, te[r], viol[r], rr[r])
+
+
+def test_ties_and_degenerate_inputs(S):
+    # simultaneous arrivals, arrival exactly at a block end, one-block models, one request
+    blocks = [[5, 5, 5], [2], [7]]
+    arr = np.array([[0, 0, 5, 5, 10, 17, 17, 30]], dtype=np.int64)
+    ty = np.array([[0, 1, 1, 2, 0, 1, 1, 2]], dtype=np.int32)
+    for pol in (Q.FIFO, Q.ALG1):
+        te, viol, rr = _run(S, blocks, arr, ty, pol)
+        _check_replica(blocks, arr[0], ty[0], pol, te[0], viol[0], rr[0])
+    te, viol, rr = _run(S, [[5, 5, 5], [2]], np.array([[0, 1]], dtype=np.int64), np.array([[0, 1]], dtype=np.int32),
+                        Q.ALG1, [1000, 2000, 3000])
+    assert te[0].tolist() == [17, 6]          # the worked example of tests/test_oracle_qos.py
+    assert viol[0].tolist() == [2, 1, 0]
+    te, _, _ = _run(S, [[4]], np.array([[3]], dtype=np.int64), np.array([[0]], dtype=np.int32), Q.ALG1)
+    assert te.tolist() == [[4]]
+
+
+def test_table2_sized_run_sampled(S):
+    # Table 2's heaviest scenario (lambda = 110 ms), 1000 requests, five models whose
+    # blocks come from 4-way splits of the paper-five chains' totals
+    tot = [10_800_000, 13_200_000, 28_350_000, 67_500_000, 20_400_000]
+    rng = np.random.default_rng(11)
+    blocks = []
+    for T in tot:
+        w = rng.uniform(0.8, 1.2, size=4)
+        b = np.floor(T * w / w.sum()).astype(np.int64)
+        blocks.append([int(x) for x in b])
+    arr, ty = wl.qos_requests(8192, 1000, 110_000_000, 5, seed=7)
+    for pol in (Q.FIFO, Q.ALG1):
+        te, viol, rr = _run(S, blocks, arr, ty, pol)
+        ext = np.array([sum(b) for b in blocks], dtype=np.int64)
+        assert (te >= ext[ty]).all()                                # never faster than isolated
+        assert (np.diff(viol[:, :19].astype(np.int64), axis=1) <= 0).all()   # monotone in alpha
+        for r in (0, 4095, 8191):
+            _check_replica(blocks, arr[r], ty[r], pol, te[r], viol[r], rr[r])
+
+
+def test_error_paths(S):
+    blocks = [[5]]
+    a = torch.tensor([[5, 3]], dtype=torch.int64, device="cuda")          # arrivals out of order
+    t = torch.zeros((1, 2), dtype=torch.int32, device="cuda")
+    with pytest.raises(S.SplitError) as e:
+        S.split_qos_simulate(blocks, a, t, [2000], 1)
+    assert e.value.code == S.SPLIT_E_RANGE
+    a = torch.zeros((1, 40), dtype=torch.int64, device="cuda")            # 40 simultaneous: > 32 pending
+    t = torch.zeros((1, 40), dtype=torch.int32, device="cuda")
+    with pytest.raises(S.SplitError) as e:
+        S.split_qos_simulate(blocks, a, t, [2000], 0)
+    assert e.value.code == S.SPLIT_E_RANGE
+    with pytest.raises(S.SplitError) as e:
+        S.split_qos_simulate([[0]], a, t, [2000], 0)                        # zero-length block
+    assert e.value.code == S.SPLIT_E_RANGE
