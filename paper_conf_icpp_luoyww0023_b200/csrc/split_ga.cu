@@ -1042,6 +1042,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const uint32_t chunks = (nchild + 31u) / 32u;
     const uint32_t first = warp * a.cpi + wl;
+    const uint64_t tau = __ldcg(tau_ptr);     // lagged elite threshold: stable during this phase
     for (uint32_t cidx_ = first; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
         const uint32_t base = cidx_ * 32u;
         const uint32_t t = base + lane;
@@ -1081,7 +1082,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         if (tr) a.trace[(g - a.g_begin) * 16 + 11] = gtimer() + 0 * (uint64_t)__double_as_longlong(f);
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
-        append_if(fkey(f) > __ldcg(tau_ptr), s_ccnt, ckey, cidx, fkey(f), slot);
+        append_if(fkey(f) > tau, s_ccnt, ckey, cidx, fkey(f), slot);
         if (tr) a.trace[(g - a.g_begin) * 16 + 14] = gtimer();
         // a8 filter: only children that beat a snapshot of an earlier record of this
         // island (a lower bound of the current record) can change the record
@@ -1310,8 +1311,6 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
                                a.tau + tau_par * I + i, sm.misc + 24, a.cand_key[Lb] + reg, a.cand_idx[Lb] + reg,
                                a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre,
                                have_fpre ? fpre : nullptr);
-            // snapshot for breed(g+1), read before the barrier: REC(g-1) (parity of g+1),
-            // stable during this phase and a lower bound of every later record
             snap = load_snapshot<WT>(a, i, nxt);
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();
@@ -1324,6 +1323,8 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
                 a.cand_cnt[((size_t)Lb * I + my_island) * cpp + my_local] = sm.misc[24];
                 sm.misc[24] = 0;
             }
+            if (kTrace && a.trace && g - a.g_begin >= 40 && g - a.g_begin < 40 + kTraceArrGens)
+                a.trace[a.trace_gens * 16 + (g - a.g_begin - 40) * 1024 + blockIdx.x] = gtimer();
             asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(a.gbar) : "memory");
         }
         if (worker) precompute_draws(a, my_island, g, my_local, pre, have_pre);

@@ -11,6 +11,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <string>
 #include <new>
 #include <vector>
 
@@ -481,7 +482,7 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     plan.add(&h->d_recpack, (size_t)a.I_total * (h->W + 2));
     if (getenv("SPLIT_TRACE")) {
         h->trace_gens = 64;
-        plan.add(&h->d_trace, (size_t)h->trace_gens * 16);
+        plan.add(&h->d_trace, (size_t)h->trace_gens * 16 + kTraceArrGens * 1024);   // + per-CTA arrivals
     }
     TRY(commit_plan(h, plan));
     ch.po = (const uint2*)d_po;
@@ -747,7 +748,7 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     h->last_gen = gens_run;
     h->have_pop = true;
     if (h->d_trace) {
-        std::vector<unsigned long long> tr((size_t)h->trace_gens * 16);
+        std::vector<unsigned long long> tr((size_t)h->trace_gens * 16 + kTraceArrGens * 1024);
         CU(cudaMemcpy(tr.data(), h->d_trace, tr.size() * 8, cudaMemcpyDeviceToHost));
         if (FILE* f = fopen(getenv("SPLIT_TRACE"), "w")) {
             fprintf(f, "gen,lead_start,lead_record,lead_sort,lead_end,work_start,work_end,lead_sync,work_sync,"
@@ -759,6 +760,16 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
                 fprintf(f, "\n");
             }
             fclose(f);
+            // per-CTA arrival instants of kTraceArrGens generations: <path>.arrivals
+            std::string p2 = std::string(getenv("SPLIT_TRACE")) + ".arrivals";
+            if (FILE* f2 = fopen(p2.c_str(), "w")) {
+                for (uint32_t g = 0; g < kTraceArrGens; ++g) {
+                    fprintf(f2, "%u", g);
+                    for (int c = 0; c < h->grid; ++c) fprintf(f2, ",%llu", tr[(size_t)h->trace_gens * 16 + g * 1024 + c]);
+                    fprintf(f2, "\n");
+                }
+                fclose(f2);
+            }
         }
     }
     if (fchk != best.f) return fail(SPLIT_E_STATE, "best record fitness mismatch (internal)");

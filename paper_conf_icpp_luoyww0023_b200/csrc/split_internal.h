@@ -11,6 +11,7 @@ constexpr uint32_t kMaxElite = 1024;        // E and K (v1 bound)
 constexpr uint32_t kCandCap = 2048;         // fast elite merge handles up to this many candidates
 constexpr uint32_t kRecWin = 256;           // record-candidate entries staged by TMA
 constexpr uint32_t kMaxWords = 64;          // n_ops <= 4097
+constexpr uint32_t kTraceArrGens = 8;       // SPLIT_TRACE: generations whose per-CTA arrivals are kept
 constexpr uint32_t kBlock = 512;            // threads per CTA of the GA kernel (one CTA per SM)
 
 enum Tag : uint32_t { TAG_INIT = 1, TAG_SELECT = 2, TAG_XOVER = 3, TAG_MUTATE = 4, TAG_REPAIR = 5 };

@@ -14,7 +14,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libsplit_ga.so")
+LIB_PATH = os.environ.get("SPLIT_LIB") or os.path.join(_PKG, "lib", "libsplit_ga.so")   # SPLIT_LIB: tuning A/B only
 
 SPLIT_OK = 0
 SPLIT_E_INVAL, SPLIT_E_RANGE, SPLIT_E_ALIGN, SPLIT_E_NOMEM, SPLIT_E_CUDA, SPLIT_E_NCCL, SPLIT_E_STATE = range(-1, -8, -1)

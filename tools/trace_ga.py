@@ -49,8 +49,25 @@ def show(path):
     print(f"{'generation (worker sync to sync)':32s} median {per[len(per) // 2] / 1e3:7.2f} us")
 
 
+def arrivals(path):
+    """Per-CTA arrival spread at the generation barrier (SPLIT_TRACE=<p> writes <p>.arrivals)."""
+    rows = [list(map(int, ln.split(","))) for ln in open(path) if ln.strip()]
+    for r in rows:
+        t = [x for x in r[1:] if x]
+        if not t:
+            continue
+        lo = min(t)
+        d = sorted((x - lo, c) for c, x in enumerate(r[1:]) if x)
+        lead = r[1] - lo
+        print(f"gen {r[0]}: leader arrives +{lead / 1e3:.2f} us; workers median +{d[len(d) // 2][0] / 1e3:.2f}, "
+              f"p90 +{d[int(len(d) * 0.9)][0] / 1e3:.2f}, last +{d[-1][0] / 1e3:.2f} us (CTA {d[-1][1]}); "
+              f"slowest 5: {[c for _, c in d[-5:]]}")
+
+
 if __name__ == "__main__":
     if sys.argv[1] == "run":
         run()
+    elif sys.argv[1] == "arrivals":
+        arrivals(sys.argv[2])
     else:
         show(sys.argv[2])
