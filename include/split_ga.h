@@ -159,10 +159,12 @@ int split_preempt_decide(const split_queue_state* q, uint32_t* insert_pos);
  *   blocks_ns    host, sum(n_blocks) entries: model m's blocks in order, each in
  *                [1, 2^32); Ext(m) = sum of its blocks < 2^32
  *   n_blocks     host, n_types entries (1..65535); n_types in [1, 65535]
- *   arrival_ns   device int64 [n_rep][n_req], non-decreasing per replica, >= 0
- *   type_id      device uint32 [n_rep][n_req], < n_types
+ *   arrival_ns   device int64 [n_req][n_rep] (request-major: request i of replica
+ *                r at i*n_rep + r, so a warp's accesses coalesce), non-decreasing
+ *                over i per replica, >= 0
+ *   type_id      device uint32 [n_req][n_rep], < n_types
  *   alpha_milli  host, n_alpha (<= 32) thresholds alpha*1000 (> 0)
- *   t_ete_out    device int64 [n_rep][n_req]: end-to-end latency per request
+ *   t_ete_out    device int64 [n_req][n_rep]: end-to-end latency per request
  *   viol_out     device uint32 [n_rep][n_alpha]: #{i : 1000 t_ete > alpha_milli Ext}
  *   rr_out       device double [n_rep][2]: sum of t_ete/Ext and of its square,
  *                added in request order

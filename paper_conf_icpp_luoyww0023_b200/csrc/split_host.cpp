@@ -1078,9 +1078,14 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
     a.viol = viol_out;
     a.rr = rr_out;
     if (qos_smem_bytes(a) > 227 * 1024) return fail(SPLIT_E_INVAL, "split_qos_simulate: model tables too large");
-    DevScratch sc;
-    uint32_t* d_tab;
-    RC(sc.alloc(&d_tab, tab.size()));
+    // stream-ordered scratch (no device-wide synchronisation in cudaFree)
+    uint32_t* d_tab = nullptr;
+    CU(cudaMallocAsync((void**)&d_tab, tab.size() * 4, st));
+    struct FreeAsync {
+        void* p;
+        cudaStream_t s;
+        ~FreeAsync() { cudaFreeAsync(p, s); }
+    } guard{d_tab, st};
     CU(cudaMemcpyAsync(d_tab, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice, st));
     a.blk_off = d_tab;
     a.ext = d_tab + n_types + 1;

@@ -111,7 +111,7 @@ struct ExhArgs {
 size_t exh_smem_bytes(const ExhArgs& a);
 int exh_blocks_per_sm(const ExhArgs& a);
 // f2 QoS simulator (split_qos.cu)
-constexpr uint32_t kQosThreads = 128;   // replicas per CTA (one per thread)
+constexpr uint32_t kQosThreads = 64;    // replicas per CTA (one per thread): 7 CTAs per SM fit 65,536 replicas in one wave
 constexpr uint32_t kQosQueue = 32;      // pending requests a replica may hold
 constexpr uint32_t kQosMaxAlpha = 32;
 struct QosArgs {
@@ -122,9 +122,9 @@ struct QosArgs {
     const uint32_t* alpha_milli;   // [n_alpha]
     uint64_t n_rep;
     uint32_t n_req;
-    const int64_t* arrival;        // [n_rep][n_req]
-    const uint32_t* type;          // [n_rep][n_req]
-    int64_t* t_ete;                // [n_rep][n_req]
+    const int64_t* arrival;        // [n_req][n_rep] (request-major)
+    const uint32_t* type;          // [n_req][n_rep]
+    int64_t* t_ete;                // [n_req][n_rep]
     uint32_t* viol;                // [n_rep][n_alpha]
     double* rr;                    // [n_rep][2]
     uint32_t* err;                 // 0 ok, 1 bad arrival/type, 2 queue overflow

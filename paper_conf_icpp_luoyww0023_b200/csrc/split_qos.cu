@@ -9,7 +9,9 @@
 // the two sums of response ratios (Eq. 3) are IEEE doubles added in request
 // order, so results are bit-identical to oracle/qos.py.
 //
-// Layout: the pending queue of each thread lives in shared memory in SoA form
+// Layout: request streams are request-major (element [i][r] of replica r at
+// i * n_rep + r), so a warp's loads and stores of request i are coalesced; the
+// pending queue of each thread lives in shared memory in SoA form
 // q[j][tid] (entry j of thread tid at j * kQosThreads + tid: conflict-free),
 // the model tables (block offsets, block ns, Ext per type) and the alpha list
 // are staged once per CTA.
@@ -38,9 +40,10 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + tid;
     if (r >= a.n_rep) return;
     const uint32_t n_req = a.n_req;
-    const int64_t* arr = a.arrival + r * n_req;
-    const uint32_t* ty = a.type + r * n_req;
-    int64_t* te = a.t_ete + r * n_req;
+    const uint64_t st = a.n_rep;                          // request-major stride
+    const int64_t* arr = a.arrival + r;
+    const uint32_t* ty = a.type + r;
+    int64_t* te = a.t_ete + r;
 #define Q(arr_, j) arr_[(j) * kQosThreads + tid]
     uint32_t n = 0, i = 0, done = 0;
     bool idle = true, run_last = false;
@@ -57,7 +60,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
         const uint32_t b = s_blk[s_off[m] + blk];
         const uint32_t left = Q(q_left, 0) - b;
         run_req = Q(q_req, 0);
-        run_arr = __ldg(arr + run_req);
+        run_arr = __ldg(arr + run_req * st);
         busy = now + b;
         idle = false;
         run_last = (left == 0u);
@@ -77,7 +80,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
         if (!idle && (i >= n_req || busy < next_a)) {
             now = busy;                                   // block end
             if (run_last) {
-                __stcs(te + run_req, now - run_arr);
+                __stcs(te + run_req * st, now - run_arr);
                 ++done;
             }
             idle = true;
@@ -110,8 +113,8 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
             ++n;
             ++i;
             if (i < n_req) {
-                next_a = __ldcs(arr + i);
-                next_t = __ldcs(ty + i);
+                next_a = __ldcs(arr + i * st);
+                next_t = __ldcs(ty + i * st);
             }
             dispatch();
         }
@@ -125,8 +128,8 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     for (uint32_t j = 0; j < a.n_alpha; ++j) s_viol[j * kQosThreads + tid] = 0;
     double rs = 0.0, rq = 0.0;
     for (uint32_t k = 0; k < n_req; ++k) {
-        const int64_t t = __ldcs(te + k);
-        const uint32_t e = s_ext[__ldcs(ty + k)];
+        const int64_t t = __ldcs(te + k * st);
+        const uint32_t e = s_ext[__ldcs(ty + k * st)];
         const uint64_t t1000 = 1000ull * (uint64_t)t;
         for (uint32_t j = 0; j < a.n_alpha; ++j)
             s_viol[j * kQosThreads + tid] += (t1000 > (uint64_t)s_alpha[j] * e) ? 1u : 0u;

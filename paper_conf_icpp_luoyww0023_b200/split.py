@@ -144,16 +144,17 @@ def split_preempt_decide(now_ns: int, alpha: float, queue, incoming) -> int:
 
 def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int = 0, stream=None):
     """f2 QoS simulator (include/split_ga.h).  blocks: per model type, its block
-    times (ns); arrival: device int64 tensor [n_rep, n_req]; type_id: device int32
-    tensor of the same shape.  Returns device tensors (t_ete [n_rep, n_req] int64,
-    violations [n_rep, n_alpha] int32 (uint32 bits), rr [n_rep, 2] f64)."""
+    times (ns); arrival: device int64 tensor [n_req, n_rep] (request-major);
+    type_id: device int32 tensor of the same shape.  Returns device tensors
+    (t_ete [n_req, n_rep] int64, violations [n_rep, n_alpha] int32 (uint32 bits),
+    rr [n_rep, 2] f64)."""
     import torch
-    n_rep, n_req = arrival.shape
+    n_req, n_rep = arrival.shape
     flat = np.ascontiguousarray(np.concatenate([np.asarray(b, dtype=np.int64) for b in blocks]))
     nb = np.ascontiguousarray(np.array([len(b) for b in blocks], dtype=np.uint32))
     al = np.ascontiguousarray(np.asarray(alpha_milli, dtype=np.uint32))
     dev = arrival.device
-    t_ete = torch.empty((n_rep, n_req), dtype=torch.int64, device=dev)
+    t_ete = torch.empty((n_req, n_rep), dtype=torch.int64, device=dev)
     viol = torch.empty((n_rep, max(len(al), 1)), dtype=torch.int32, device=dev)
     rr = torch.empty((n_rep, 2), dtype=torch.float64, device=dev)
     assert arrival.dtype == torch.int64 and arrival.is_contiguous()

@@ -216,7 +216,8 @@ def qos_requests(n_rep: int, n_req: int, lam_ns: int, n_types: int, seed: int):
     mean arrival interval lambda, here in ns): per replica, exponential
     inter-arrival gaps rounded to integer ns (cumulative, starting at the first
     gap) and a model type uniform in [0, n_types).  Returns (arrival int64
-    [n_rep, n_req], type int32 [n_rep, n_req])."""
+    [n_rep, n_req], type int32 [n_rep, n_req]), replica-major; the simulator
+    takes the request-major transposes (np.ascontiguousarray(x.T))."""
     rng = np.random.default_rng(seed)
     gaps = np.rint(rng.exponential(float(lam_ns), size=(n_rep, n_req))).astype(np.int64)
     arrival = np.cumsum(gaps, axis=1)

@@ -25,11 +25,12 @@ def S():
 
 
 def _run(S, blocks, arr, ty, policy, alphas=ALPHAS):
-    a = torch.from_numpy(arr).cuda()
-    t = torch.from_numpy(ty).cuda()
+    # replica-major in the tests, request-major at the ABI
+    a = torch.from_numpy(np.ascontiguousarray(arr.T)).cuda()
+    t = torch.from_numpy(np.ascontiguousarray(ty.T)).cuda()
     te, viol, rr = S.split_qos_simulate(blocks, a, t, alphas, policy)
     torch.cuda.synchronize()
-    return te.cpu().numpy(), viol.cpu().numpy().view(np.uint32), rr.cpu().numpy()
+    return np.ascontiguousarray(te.cpu().numpy().T), viol.cpu().numpy().view(np.uint32), rr.cpu().numpy()
 
 
 def _check_replica(blocks, arr, ty, policy, te, viol, rr, alphas=ALPHAS):
@@ -90,13 +91,13 @@ def test_table2_sized_run_sampled(S):
 
 def test_error_paths(S):
     blocks = [[5]]
-    a = torch.tensor([[5, 3]], dtype=torch.int64, device="cuda")          # arrivals out of order
-    t = torch.zeros((1, 2), dtype=torch.int32, device="cuda")
+    a = torch.tensor([[5], [3]], dtype=torch.int64, device="cuda")        # arrivals out of order
+    t = torch.zeros((2, 1), dtype=torch.int32, device="cuda")
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate(blocks, a, t, [2000], 1)
     assert e.value.code == S.SPLIT_E_RANGE
-    a = torch.zeros((1, 40), dtype=torch.int64, device="cuda")            # 40 simultaneous: > 32 pending
-    t = torch.zeros((1, 40), dtype=torch.int32, device="cuda")
+    a = torch.zeros((40, 1), dtype=torch.int64, device="cuda")            # 40 simultaneous: > 32 pending
+    t = torch.zeros((40, 1), dtype=torch.int32, device="cuda")
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate(blocks, a, t, [2000], 0)
     assert e.value.code == S.SPLIT_E_RANGE

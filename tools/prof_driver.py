@@ -1,5 +1,5 @@
 """Minimal drivers for ncu captures (one GPU): `eval` runs split_eval_batch on C5,
-`ga` runs split_ga_run on C2.  Not a benchmark (numbers under ncu are not bench values)."""
+`ga` runs split_ga_run on C2, `qos` the f2 simulator.  Not a benchmark (numbers under ncu are not bench values)."""
 import os
 import sys
 
@@ -23,6 +23,17 @@ def main(what: str, reps: int = 3, gens: int = 500):
         for _ in range(reps):
             h.eval_batch(bits, n_cand, out)
         torch.cuda.synchronize()
+    elif what == "qos":
+        blocks = [[3_575_000, 3_031_000, 3_231_000, 3_191_000], [4_005_000, 4_052_000, 3_984_000, 4_040_000],
+                  [8_984_000, 8_747_000, 8_865_000, 8_990_000], [22_314_000, 21_125_000, 18_922_000, 19_467_000],
+                  [6_124_000, 6_154_000, 6_078_000, 6_139_000]]
+        arr, typ = wl.qos_requests(65536, 1000, 110_000_000, 5, seed=2023)
+        da = torch.from_numpy(np.ascontiguousarray(arr.T)).cuda()
+        dt = torch.from_numpy(np.ascontiguousarray(typ.T)).cuda()
+        for _ in range(reps):
+            S.split_qos_simulate(blocks, da, dt, [1000 * a for a in range(2, 21)], 1)
+        torch.cuda.synchronize()
+        return
     else:
         lat, ovh = wl.chain("resnet50_175")
         h = S.SplitGA(lat, ovh, pop_size=65536, n_elite=1024, k_min=2, k_max=32, stream=st)

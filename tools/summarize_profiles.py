@@ -21,6 +21,9 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
         "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
         "sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_active", "smsp__inst_executed.sum",
+        "smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio",
+        "smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio",
+        "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
         "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
         "launch__shared_mem_per_block_dynamic"]
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-3, "nsecond": 1e-3, "us": 1.0,
@@ -74,7 +77,8 @@ def main(tag):
     md = [launches(tag)]
     traffic = {}
     for name, rep, per in (("ga_kernel", "prof_ga.ncu-rep", "launch (one RUN segment = 500 generations of C2)"),
-                           ("eval_batch_kernel", "prof_eval.ncu-rep", "launch (C5, 2^24 candidates)")):
+                           ("eval_batch_kernel", "prof_eval.ncu-rep", "launch (C5, 2^24 candidates)"),
+                           ("qos_kernel", "prof_qos.ncu-rep", "launch (f2: 65,536 replicas x 1000 requests)")):
         path = os.path.join(OUT, rep)
         if not os.path.exists(path):
             continue
