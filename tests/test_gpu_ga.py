@@ -164,3 +164,18 @@ def test_islands_through_nccl_communicator(S):
     assert r["generation_found"] == o["generation_found"]
     for i in range(4):
         assert np.array_equal(pops[i][0], o["population"][i])
+
+
+def test_large_population_several_chunks_per_warp(S):
+    """N = 262,144 on the BERT-base chain (W = 7, register rows of 8 words): every
+    worker warp breeds several 32-child chunks per generation (the large-N loop
+    that the C4-shaped bench island runs), compared bit for bit."""
+    lat, ovh = wl.chain("bert_base")
+    run_both(S, lat, ovh, 2, 42, pop_size=262144, n_elite=1024, k_min=2, k_max=32)
+
+
+def test_hbm_regime_island_first_generation(S):
+    """The bench's `ga_hbm_regime` configuration itself (N = 4,194,304, W = 7):
+    generation 0 and one transition, whole population bit for bit."""
+    lat, ovh = wl.chain("bert_base")
+    run_both(S, lat, ovh, 1, 77, pop_size=1 << 22, n_elite=1024, k_min=2, k_max=32)
