@@ -359,6 +359,30 @@ def main():
                          "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
                          "traffic": _profile_traffic("eval_batch_kernel_c5"),
                          "algorithmic_bytes_per_candidate": bpc}}
+        # C5 population sweep (BASELINE configs[4]: 1K-64M candidates): the 2^24 rows tiled on the device
+        sweep = []
+        for lg in (10, 14, 18, 22, 24, 26):
+            n = 1 << lg
+            if n <= C5_EVAL_N:
+                b_n = bits[:n]
+            else:
+                b_n = bits.repeat(n // C5_EVAL_N, 1)
+            f_n = torch.empty(n, dtype=torch.float64, device=dev)
+            h5.eval_batch(b_n, n, f_n)
+            reps = 5 if lg >= 22 else 50
+            z0, z1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            z0.record(stream)
+            for _ in range(reps):
+                h5.eval_batch(b_n, n, f_n)
+            z1.record(stream)
+            torch.cuda.synchronize()
+            zms = z0.elapsed_time(z1) / reps
+            zg = bpc * n / (zms / 1000.0) / 1e9
+            sweep.append({"n_cand": n, "ms": zms, "evals_per_s": n / (zms / 1000.0), "gbs": zg,
+                          "frac": zg / peaks["hbm_gbs"], "l2_resident": bpc * n < 100e6})
+            del b_n, f_n
+        out["eval_batch"]["sweep"] = sweep
         h5.close()
         del bits, fout
 

@@ -48,10 +48,18 @@ def launches(tag):
         agg[d["Kernel Name"].split("(")[0]][1] += us
     tot = sum(v[1] for v in agg.values())
     lines = [f"# Launch list ({tag}): `ncu --metrics gpu__time_duration.sum --clock-control none` over "
-             "`bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-e2e` (cold-cache, serialised: compare shares)", "",
+             "`bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-ga-big --no-qos` (cold-cache, serialised: "
+             "compare shares; includes the eval_batch and f1 sub-measurements)", "",
              "| kernel | launches | total us | share |", "|---|---|---|---|"]
     for k, v in sorted(agg.items(), key=lambda x: -x[1][1]):
         lines.append(f"| `{k}` | {v[0]} | {v[1]:.1f} | {100 * v[1] / tot:.1f}% |")
+    # the headline step (one split_ga_run) only: its kernels' shares
+    step = {k: v for k, v in agg.items() if "ga_kernel" in k or "eval_stats_kernel" in k}
+    st = sum(v[1] for v in step.values()) or 1.0
+    lines += ["", "GA step only (split_ga_run: INIT + RUN launches and the best-record statistics kernel):", "",
+              "| kernel | launches | total us | share of step |", "|---|---|---|---|"]
+    for k, v in sorted(step.items(), key=lambda x: -x[1][1]):
+        lines.append(f"| `{k}` | {v[0]} | {v[1]:.1f} | {100 * v[1] / st:.1f}% |")
     shutil.copy(path, os.path.join(PROF, f"{tag}_launches.csv"))
     return "\n".join(lines) + "\n"
 
