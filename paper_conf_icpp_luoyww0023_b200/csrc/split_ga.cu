@@ -154,12 +154,62 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uin
     return eq2(k, V, OV, ch);
 }
 
+// Wide rows (4 < W <= 16): the row's 32-bit halves go to this thread's slot of
+// shared memory (odd pitch 2W+1: conflict-free), then one loop iteration per
+// cut, descending, refilling from the occupancy mask -- the trip count is the
+// child's cut count, not a per-word maximum over the warp's lanes.  Same
+// integer statistics and Eq. 2 tail as eval_walk (R3, R5').
+template <int WT>
+__device__ __forceinline__ double eval_wide(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
+                                            const Row<WT>& r, uint32_t* my)
+{
+    uint32_t occ = 0, cuts = 0;
+#pragma unroll
+    for (int i = 0; i < WT; ++i) {
+        if (i < (int)ch.W) {
+            const uint64_t wv = r.w[i] & word_mask(ch, i);
+            const uint32_t lo = (uint32_t)wv, hi = (uint32_t)(wv >> 32);
+            my[2 * i] = lo;
+            my[2 * i + 1] = hi;
+            occ |= ((lo != 0u ? 1u : 0u) | (hi != 0u ? 2u : 0u)) << (2 * i);
+            cuts += __popc(lo) + __popc(hi);
+        }
+    }
+    const uint32_t k = cuts + 1;
+    if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
+    uint32_t endP = ch.T, OV = 0, v = 0, qb = 0;
+    uint64_t S2 = 0;
+    for (uint32_t j = 0; j < cuts; ++j) {
+        if (v == 0u) {
+            const uint32_t q = bfind32(occ);
+            occ ^= 1u << q;
+            v = my[q];
+            qb = q << 5;
+        }
+        const uint32_t bt = bfind32(v);
+        v ^= 1u << bt;
+        const uint32_t p = qb + bt;
+        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+        const uint32_t Pp = sP[p + 1], op = sO[p];
+        const uint32_t t = endP - Pp + op;
+        S2 += (uint64_t)t * t;
+        OV += op;
+        endP = Pp;
+    }
+    S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
+    const uint64_t S1 = (uint64_t)ch.T + OV;
+    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+    return eq2(k, V, OV, ch);
+}
+
 template <int WT>
 __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
-                                            const Row<WT>& r, Stats* st)
+                                            const Row<WT>& r, Stats* st, uint32_t* srow = nullptr)
 {
     if constexpr (WT <= 4) {
         if (!st) return eval_regs_narrow<WT>(ch, sP, sO, r);
+    } else if constexpr (WT <= 16) {
+        if (!st && srow) return eval_wide<WT>(ch, sP, sO, r, srow);
     }
     // same arithmetic as eval_walk, with the word loop unrolled over the register row
     uint32_t cuts = 0;
@@ -419,6 +469,7 @@ struct Smem {
     double* pf;           // [cpi_pad] staged partial bests (leader)
     uint32_t* pi;
     uint64_t* pb;         // [cpi_pad][W] when a.stage_bits
+    uint32_t* rows;       // [kBlock][2W+1] per-thread row halves for the wide-row walk (4 < W <= 16)
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
@@ -447,6 +498,7 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take((size_t)a.cpi_pad * 8); if (s) s->pf = (double*)p;
     p = take(((size_t)a.cpi_pad + 4) * 4); if (s) s->pi = (uint32_t*)p;
     p = take(a.stage_bits ? (size_t)a.cpi_pad * a.ch.W * 8 : 16); if (s) s->pb = (uint64_t*)p;
+    p = take((a.ch.W > 4 && a.ch.W <= 16) ? (size_t)kBlock * (2 * a.ch.W + 1) * 4 : 16); if (s) s->rows = (uint32_t*)p;
     return off;
 }
 
@@ -1034,7 +1086,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
                                                const uint64_t* tau_ptr, uint32_t* s_ccnt, uint64_t* ckey,
                                                uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx,
                                                const BestRow<WT>& snap, ChildDraws& pre, bool& have_pre,
-                                               const double* fpre)
+                                               const double* fpre, uint32_t* srow)
 {
     const ChainDev& ch = a.ch;
     const uint32_t W = ch.W, N = a.N, E = a.E;
@@ -1078,7 +1130,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         if ((uint64_t)dr.mu.x < a.thr_m) row_xor_bit(A, below(dr.mu.y, ch.n - 1));      // a6
         repair(a, A, gid, g);                                                              // a7
         if (tr) a.trace[(g - a.g_begin) * 16 + 10] = gtimer() + 0 * A.w[0];
-        const double f = eval_regs(ch, sP, sO, A, nullptr);                               // a2
+        const double f = eval_regs(ch, sP, sO, A, nullptr, srow);                         // a2
         if (tr) a.trace[(g - a.g_begin) * 16 + 11] = gtimer() + 0 * (uint64_t)__double_as_longlong(f);
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
@@ -1153,7 +1205,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
                 if (c >= N) continue;
                 Row<WT> r;
                 init_row(a, r, (a.island_base + i) * N + c);
-                const double f = eval_regs(a.ch, sP, sO, r, nullptr);
+                const double f = eval_regs(a.ch, sP, sO, r, nullptr, sm.rows + threadIdx.x * (2 * W + 1));
                 row_store(r, pop + (size_t)c * W, W);
                 fit[c] = f;
                 track_row(best, f, c, r, W);
@@ -1310,7 +1362,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
                                a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
                                a.tau + tau_par * I + i, sm.misc + 24, a.cand_key[Lb] + reg, a.cand_idx[Lb] + reg,
                                a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre,
-                               have_fpre ? fpre : nullptr);
+                               have_fpre ? fpre : nullptr, sm.rows + threadIdx.x * (2 * W + 1));
             snap = load_snapshot<WT>(a, i, nxt);
             if (kTrace && threadIdx.x == 0 && blockIdx.x == I && a.trace && g - a.g_begin < a.trace_gens)
                 a.trace[(g - a.g_begin) * 16 + 5] = gtimer();

@@ -34,6 +34,11 @@ def main(what: str, reps: int = 3, gens: int = 500):
             S.split_qos_simulate(blocks, da, dt, [1000 * a for a in range(2, 21)], 1)
         torch.cuda.synchronize()
         return
+    elif what == "ga_big":
+        lat, ovh = wl.chain("bert_base")
+        h = S.SplitGA(lat, ovh, pop_size=1 << 22, n_elite=1024, k_min=2, k_max=32, stream=st)
+        for i in range(reps):
+            h.run(gens, i)
     else:
         lat, ovh = wl.chain("resnet50_175")
         h = S.SplitGA(lat, ovh, pop_size=65536, n_elite=1024, k_min=2, k_max=32, stream=st)
