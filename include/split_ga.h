@@ -198,6 +198,15 @@ void split_comm_destroy(void* comm);
  * handle's stream; device scratch is allocated and freed inside the call. */
 int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* min_v_per_k, uint64_t* argmin_per_k);
 
+/* a0 again on a live handle: replace its chain (same n_ops) -- new per-operator
+ * latencies and cut overheads (host, copied; NULL overheads = 0), validated and
+ * guarded exactly as split_ga_create does for the handle's k_max -- and upload
+ * the tables stream-ordered on the handle's stream.  No allocation: the serving
+ * path re-splits a model whose profile changed without create/destroy.  The
+ * population is invalidated (split_ga_run re-initialises anyway).
+ * SPLIT_E_INVAL / SPLIT_E_RANGE as in split_ga_create. */
+int split_ga_set_chain(split_ga_t* h, const int64_t* latencies_ns, const int64_t* cut_overhead_ns);
+
 /* f1 — minimum S2 = sum t_j^2 over all k-block splits, k = 1..k_max, by the
  * O(k n^2) dynamic program D[j][i] = min_p D[j-1][p] + (P[i]-P[p]+ovh[p-1])^2
  * (one CTA on the handle's device).  Exact for any per-cut overheads; with a

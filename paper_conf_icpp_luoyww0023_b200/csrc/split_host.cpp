@@ -286,17 +286,72 @@ static uint32_t pow2_at_least(uint32_t x)
         }                       \
     } while (0)
 
-extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_params* pp, split_ga_t** out)
+// a0: host tables of one chain -- P and ovh words, the {P[p+1], ovh[p]} pairs, the
+// Eq. 2 reciprocals -- after validation and the exact-integer guards for k_max.
+struct ChainHost {
+    std::vector<uint32_t> words, po;
+    std::vector<double> rcp;
+    uint32_t p_words = 0, o_words = 0;
+    uint64_t T = 0;
+};
+
+static int chain_tables(const int64_t* lat, const int64_t* ovh_in, uint32_t n, uint32_t k_max, ChainHost& c)
 {
-    if (!lat || !pp || !out) return fail(SPLIT_E_INVAL, "split_ga_create: NULL argument");
-    const split_ga_params p = *pp;
-    if (n < 2 || n > 64u * kMaxWords + 1) return fail(SPLIT_E_INVAL, "n_ops must be in [2, %u]", 64u * kMaxWords + 1);
     unsigned __int128 T = 0;
     for (uint32_t i = 0; i < n; ++i) {
         if (lat[i] < 0) return fail(SPLIT_E_INVAL, "latencies_ns[%u] < 0", i);
         T += (uint64_t)lat[i];
     }
     if (T < 1) return fail(SPLIT_E_INVAL, "sum of latencies must be >= 1");
+    std::vector<int64_t> ovh(n - 1, 0);
+    if (ovh_in) {
+        for (uint32_t i = 0; i + 1 < n; ++i) {
+            if (ovh_in[i] < 0) return fail(SPLIT_E_INVAL, "cut_overhead_ns[%u] < 0", i);
+            ovh[i] = ovh_in[i];
+        }
+    }
+    // exact-integer guards (a0)
+    std::vector<int64_t> srt(ovh);
+    std::sort(srt.begin(), srt.end(), std::greater<int64_t>());
+    unsigned __int128 Tp = T;
+    for (uint32_t i = 0; i + 1 < k_max && i < srt.size(); ++i) Tp += (uint64_t)srt[i];
+    if (Tp >= ((unsigned __int128)1 << 32)) return fail(SPLIT_E_RANGE, "T + largest overheads must be < 2^32 ns");
+    if ((unsigned __int128)(k_max - 1) * Tp * Tp >= ((unsigned __int128)1 << 63))
+        return fail(SPLIT_E_RANGE, "(k_max-1) * T'^2 must be < 2^63");
+    // chain words: P[0..n] padded to x4, ovh[0..n-2] padded to x4
+    c.p_words = (n + 1 + 3) & ~3u;
+    c.o_words = (n - 1 + 3) & ~3u;
+    c.words.assign(c.p_words + c.o_words, 0);
+    uint64_t acc = 0;
+    for (uint32_t i = 0; i < n; ++i) {
+        c.words[i] = (uint32_t)acc;
+        acc += (uint64_t)lat[i];
+    }
+    c.words[n] = (uint32_t)acc;
+    for (uint32_t i = 0; i + 1 < n; ++i) c.words[c.p_words + i] = (uint32_t)ovh[i];
+    // interleaved {P[p+1], ovh[p]} table for the eval kernel's walk
+    const uint32_t po_n = ((n - 1) + 1) & ~1u;                  // entries, even -> 16-byte multiple
+    c.po.assign(2 * (size_t)po_n, 0);
+    for (uint32_t q = 0; q + 1 < n; ++q) {
+        c.po[2 * q] = c.words[q + 1];
+        c.po[2 * q + 1] = (uint32_t)ovh[q];
+    }
+    // Eq. 2 reciprocals (ChainDev::rcp): IEEE divisions, i.e. correctly rounded
+    c.rcp.assign(2 * (size_t)n + 2, 0.0);
+    c.rcp[0] = 1.0 / (double)acc;
+    for (uint32_t k = 1; k <= n; ++k) {
+        c.rcp[k] = 1.0 / (double)k;
+        c.rcp[n + 1 + k] = 1.0 / ((double)k * (double)acc);   // k T < 2^53: exact product
+    }
+    c.T = acc;
+    return SPLIT_OK;
+}
+
+extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_params* pp, split_ga_t** out)
+{
+    if (!lat || !pp || !out) return fail(SPLIT_E_INVAL, "split_ga_create: NULL argument");
+    const split_ga_params p = *pp;
+    if (n < 2 || n > 64u * kMaxWords + 1) return fail(SPLIT_E_INVAL, "n_ops must be in [2, %u]", 64u * kMaxWords + 1);
     if (p.pop_size < 2) return fail(SPLIT_E_INVAL, "pop_size must be >= 2");
     if (p.n_elite > p.pop_size || p.n_elite > kMaxElite) return fail(SPLIT_E_INVAL, "n_elite must be <= min(N, %u)", kMaxElite);
     if ((p.pop_size - p.n_elite) & 1u) return fail(SPLIT_E_INVAL, "pop_size - n_elite must be even");
@@ -316,21 +371,12 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     const bool migrate = p.migration_interval > 0 && p.n_islands > 1;
     if (migrate && (p.n_migrants < 1 || p.n_migrants > p.pop_size - p.n_elite || p.n_migrants > kMaxElite))
         return fail(SPLIT_E_INVAL, "n_migrants must be in [1, min(N - E, %u)]", kMaxElite);
-    std::vector<int64_t> ovh(n - 1, 0);
-    if (p.cut_overhead_ns) {
-        for (uint32_t i = 0; i + 1 < n; ++i) {
-            if (p.cut_overhead_ns[i] < 0) return fail(SPLIT_E_INVAL, "cut_overhead_ns[%u] < 0", i);
-            ovh[i] = p.cut_overhead_ns[i];
-        }
+    ChainHost chn;
+    {
+        const int rc = chain_tables(lat, p.cut_overhead_ns, n, p.k_max, chn);
+        if (rc != SPLIT_OK) return rc;
     }
-    // exact-integer guards (a0)
-    std::vector<int64_t> srt(ovh);
-    std::sort(srt.begin(), srt.end(), std::greater<int64_t>());
-    unsigned __int128 Tp = T;
-    for (uint32_t i = 0; i + 1 < p.k_max && i < srt.size(); ++i) Tp += (uint64_t)srt[i];
-    if (Tp >= ((unsigned __int128)1 << 32)) return fail(SPLIT_E_RANGE, "T + largest overheads must be < 2^32 ns");
-    if ((unsigned __int128)(p.k_max - 1) * Tp * Tp >= ((unsigned __int128)1 << 63))
-        return fail(SPLIT_E_RANGE, "(k_max-1) * T'^2 must be < 2^63");
+    const uint64_t T = chn.T;
 
     split_ga_t* h = new (std::nothrow) split_ga_t();
     if (!h) return fail(SPLIT_E_NOMEM, "host alloc");
@@ -349,36 +395,17 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
             return fail(SPLIT_E_CUDA, "device %d: %s", p.device, cudaGetErrorString(e));
         }
     }
-    // chain words: P[0..n] padded to x4, ovh[0..n-2] padded to x4
-    const uint32_t p_words = (n + 1 + 3) & ~3u, o_words = (n - 1 + 3) & ~3u;
-    std::vector<uint32_t> words(p_words + o_words, 0);
-    uint64_t acc = 0;
-    for (uint32_t i = 0; i < n; ++i) {
-        words[i] = (uint32_t)acc;
-        acc += (uint64_t)lat[i];
-    }
-    words[n] = (uint32_t)acc;
-    for (uint32_t i = 0; i + 1 < n; ++i) words[p_words + i] = (uint32_t)ovh[i];
-    // interleaved {P[p+1], ovh[p]} table for the eval kernel's walk
-    const uint32_t po_n = ((n - 1) + 1) & ~1u;                  // entries, even -> 16-byte multiple
-    std::vector<uint32_t> po(2 * (size_t)po_n, 0);
-    for (uint32_t q = 0; q + 1 < n; ++q) {
-        po[2 * q] = words[q + 1];
-        po[2 * q + 1] = (uint32_t)ovh[q];
-    }
+    std::vector<uint32_t>& words = chn.words;
+    std::vector<uint32_t>& po = chn.po;
+    std::vector<double>& rcp = chn.rcp;
+    const uint32_t p_words = chn.p_words, o_words = chn.o_words;
+    const uint64_t acc = chn.T;
     DevPlan plan;
     uint32_t* d_chain = nullptr;
     uint32_t* d_po = nullptr;
+    double* d_rcp = nullptr;
     plan.add(&d_chain, words.size());
     plan.add(&d_po, po.size());
-    // Eq. 2 reciprocals (ChainDev::rcp): IEEE divisions, i.e. correctly rounded
-    std::vector<double> rcp(2 * (size_t)n + 2, 0.0);
-    rcp[0] = 1.0 / (double)acc;
-    for (uint32_t k = 1; k <= n; ++k) {
-        rcp[k] = 1.0 / (double)k;
-        rcp[n + 1 + k] = 1.0 / ((double)k * (double)acc);   // k T < 2^53: exact product
-    }
-    double* d_rcp = nullptr;
     plan.add(&d_rcp, rcp.size());
     h->hwords = words;
     h->p_words = p_words;
@@ -501,6 +528,26 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
         if (e != cudaSuccess) TRY(fail(SPLIT_E_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
     }
     *out = h;
+    return SPLIT_OK;
+}
+
+extern "C" int split_ga_set_chain(split_ga_t* h, const int64_t* lat, const int64_t* cut_overhead_ns)
+{
+    if (!h || !lat) return fail(SPLIT_E_INVAL, "split_ga_set_chain: NULL argument");
+    ChainHost chn;
+    {
+        const int rc = chain_tables(lat, cut_overhead_ns, h->n, h->p.k_max, chn);
+        if (rc != SPLIT_OK) return rc;
+    }
+    CU(cudaSetDevice(h->device));
+    CU(cudaMemcpyAsync((void*)h->ch.words, chn.words.data(), chn.words.size() * 4, cudaMemcpyHostToDevice, h->stream));
+    CU(cudaMemcpyAsync((void*)h->ch.po, chn.po.data(), chn.po.size() * 4, cudaMemcpyHostToDevice, h->stream));
+    CU(cudaMemcpyAsync((void*)h->ch.rcp, chn.rcp.data(), chn.rcp.size() * 8, cudaMemcpyHostToDevice, h->stream));
+    h->T = chn.T;
+    h->ch.T = (uint32_t)chn.T;
+    h->ga.ch.T = (uint32_t)chn.T;
+    h->hwords = chn.words;
+    h->have_pop = false;
     return SPLIT_OK;
 }
 

@@ -74,6 +74,7 @@ def _load():
         "split_eval_batch": (C.c_int, [C.c_void_p, C.c_void_p, C.c_uint64, C.c_void_p]),
         "split_eval_batch_host": (C.c_int, [C.c_void_p, C.c_void_p, C.c_uint64, C.c_void_p]),
         "split_ga_run": (C.c_int, [C.c_void_p, C.c_uint32, C.c_uint64, P(split_best_t)]),
+        "split_ga_set_chain": (C.c_int, [C.c_void_p, P(C.c_int64), P(C.c_int64)]),
         "split_ga_population": (C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
         "split_preempt_decide": (C.c_int, [P(split_queue_state), P(C.c_uint32)]),
         "split_qos_simulate": (C.c_int, [P(C.c_int64), P(C.c_uint32), C.c_uint32, C.c_uint32, P(C.c_uint32),
@@ -103,7 +104,7 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_eval_batch_host", "split_ga_run", "split_ga_population", "split_preempt_decide",
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
-            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate")
+            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain")
 
 
 def lib():
@@ -260,6 +261,15 @@ class SplitGA:
             out = np.empty(n, dtype=np.float64)
         _check(_lib.split_eval_batch_host(self._h, _ptr(b), n, _ptr(out)), "split_eval_batch_host")
         return out
+
+    def set_chain(self, latencies_ns, cut_overhead_ns=None) -> None:
+        """Replace the handle's chain (same n_ops): host arrays, uploaded on the handle's stream."""
+        lat = np.ascontiguousarray(latencies_ns, dtype=np.int64)
+        ovh = None if cut_overhead_ns is None else np.ascontiguousarray(cut_overhead_ns, dtype=np.int64)
+        self._keep_chain = (lat, ovh)          # the copy is staged before the call returns; kept for clarity
+        _check(_lib.split_ga_set_chain(self._h, lat.ctypes.data_as(C.POINTER(C.c_int64)),
+                                       None if ovh is None else ovh.ctypes.data_as(C.POINTER(C.c_int64))),
+               "split_ga_set_chain")
 
     def run(self, generations: int, seed: int) -> dict:
         bits = np.zeros(max(self.W, 1), dtype=np.uint64)

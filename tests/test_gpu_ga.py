@@ -179,3 +179,24 @@ def test_hbm_regime_island_first_generation(S):
     generation 0 and one transition, whole population bit for bit."""
     lat, ovh = wl.chain("bert_base")
     run_both(S, lat, ovh, 1, 77, pop_size=1 << 22, n_elite=1024, k_min=2, k_max=32)
+
+
+def test_set_chain_matches_fresh_handle(S):
+    """split_ga_set_chain on a live handle == a handle created with that chain ==
+    the oracle; bad chains are rejected like split_ga_create rejects them."""
+    lat1, ovh1 = wl.chain("resnet50_175")
+    lat2, ovh2 = wl.chain("resnet50_175", overhead="const")
+    lat2 = lat2[::-1].copy()
+    kw = dict(pop_size=4096, n_elite=82, k_min=2, k_max=32)
+    with S.SplitGA(lat1, ovh1, **kw) as h:
+        h.run(5, 1)
+        h.set_chain(lat2, ovh2)
+        r = h.run(12, 7)
+        bits, fit = h.population(0)
+        with pytest.raises(S.SplitError) as e:
+            h.set_chain(-lat2, ovh2)
+        assert e.value.code == S.SPLIT_E_INVAL
+    o = oracle.ga_run(lat2, ovh2, 12, 7, want_population=True, **kw)
+    assert r["fitness"] == o["fitness"] and np.array_equal(r["bits"], o["bits"])
+    assert np.array_equal(bits, o["population"][0])
+    assert np.array_equal(_fbits(fit), _fbits(o["fitness_all"][0]))
