@@ -207,6 +207,24 @@ int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* min_v_per_k
  * SPLIT_E_INVAL / SPLIT_E_RANGE as in split_ga_create. */
 int split_ga_set_chain(split_ga_t* h, const int64_t* latencies_ns, const int64_t* cut_overhead_ns);
 
+/* f3 — Eq. 1-driven choice of the block count (R21).
+ * Runs the fixed-k GA (k_min = k_max = k, `generations`, `seed`) for every k
+ * in [k_lo, k_hi] (1 <= k_lo <= k_hi <= the handle's k_max) and reports each
+ * run's best split: Eq. 2 fitness, Eq. 1's expected wait S2/(2 S1) of a short
+ * request arriving during the model (P@17226-17827), overheads and V.
+ * *k_best = the k whose best split has the smallest Eq. 1 wait (ties -> the
+ * smaller k; 0 if no k has a feasible split).  out: host, k_hi-k_lo+1 entries.
+ * Synchronous; the handle's own k range is restored afterwards. */
+typedef struct {
+    uint32_t k;
+    double fitness;
+    double expected_wait_ns;
+    uint64_t overhead_ns;
+    int64_t var_num;
+} split_k_result;
+int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32_t generations, uint64_t seed,
+                  split_k_result* out, uint32_t* k_best);
+
 /* f1 — minimum S2 = sum t_j^2 over all k-block splits, k = 1..k_max, by the
  * O(k n^2) dynamic program D[j][i] = min_p D[j-1][p] + (P[i]-P[p]+ovh[p-1])^2
  * (one CTA on the handle's device).  Exact for any per-cut overheads; with a

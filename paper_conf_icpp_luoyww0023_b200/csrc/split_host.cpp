@@ -551,6 +551,48 @@ extern "C" int split_ga_set_chain(split_ga_t* h, const int64_t* lat, const int64
     return SPLIT_OK;
 }
 
+// f3: Eq. 1-driven choice of the block count.  Eq. 1 (P@17226-17827) gives the
+// expected wait of a short request arriving during the split model as
+// S2 / (2 S1) = (sigma^2/t_bar + t_bar) / 2; more blocks shrink t_bar but add
+// overhead to S1, so the wait has a minimum over k ("an optimal number of
+// splits exists", P@18542-18830).  One fixed-k GA run per k in [k_lo, k_hi]
+// (same seed, same generation budget), then k* = argmin of the Eq. 1 wait of
+// each run's best split (ties -> smaller k; k without a feasible split skipped).
+extern "C" int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32_t generations, uint64_t seed,
+                             split_k_result* out, uint32_t* k_best)
+{
+    if (!h || !out || !k_best) return fail(SPLIT_E_INVAL, "split_k_sweep: NULL argument");
+    if (k_lo < 1 || k_lo > k_hi || k_hi > h->p.k_max)
+        return fail(SPLIT_E_INVAL, "split_k_sweep: need 1 <= k_lo <= k_hi <= handle k_max = %u", h->p.k_max);
+    const uint32_t kmin0 = h->ch.k_min, kmax0 = h->ch.k_max;
+    std::vector<uint64_t> bits(h->W ? h->W : 1);
+    int rc = SPLIT_OK;
+    *k_best = 0;
+    double best_wait = 0.0;
+    for (uint32_t k = k_lo; k <= k_hi && rc == SPLIT_OK; ++k) {
+        h->ch.k_min = h->ch.k_max = k;
+        h->ga.ch.k_min = h->ga.ch.k_max = k;
+        split_best_t b;
+        memset(&b, 0, sizeof(b));
+        b.bits = bits.data();
+        rc = split_ga_run(h, generations, seed, &b);
+        if (rc != SPLIT_OK) break;
+        split_k_result& r = out[k - k_lo];
+        r.k = k;
+        r.fitness = b.fitness;
+        r.expected_wait_ns = b.expected_wait_ns;
+        r.overhead_ns = b.overhead_ns;
+        r.var_num = b.var_num;
+        if (b.fitness > -INFINITY && (*k_best == 0 || b.expected_wait_ns < best_wait)) {
+            *k_best = k;
+            best_wait = b.expected_wait_ns;
+        }
+    }
+    h->ch.k_min = h->ga.ch.k_min = kmin0;
+    h->ch.k_max = h->ga.ch.k_max = kmax0;
+    return rc;
+}
+
 extern "C" void split_ga_destroy(split_ga_t* h)
 {
     if (!h) return;

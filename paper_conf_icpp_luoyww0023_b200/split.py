@@ -50,6 +50,11 @@ class split_queue_state(C.Structure):
                 ("queue", C.POINTER(split_request)), ("incoming", split_request)]
 
 
+class split_k_result(C.Structure):
+    _fields_ = [("k", C.c_uint32), ("fitness", C.c_double), ("expected_wait_ns", C.c_double),
+                ("overhead_ns", C.c_uint64), ("var_num", C.c_int64)]
+
+
 class split_run_stats(C.Structure):
     _fields_ = [("launches", C.c_uint64), ("ms_total", C.c_float), ("ms_loop", C.c_float),
                 ("general_selects", C.c_uint32), ("fast_selects", C.c_uint32)]
@@ -75,6 +80,8 @@ def _load():
         "split_eval_batch_host": (C.c_int, [C.c_void_p, C.c_void_p, C.c_uint64, C.c_void_p]),
         "split_ga_run": (C.c_int, [C.c_void_p, C.c_uint32, C.c_uint64, P(split_best_t)]),
         "split_ga_set_chain": (C.c_int, [C.c_void_p, P(C.c_int64), P(C.c_int64)]),
+        "split_k_sweep": (C.c_int, [C.c_void_p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint64, P(split_k_result),
+                                    P(C.c_uint32)]),
         "split_ga_population": (C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
         "split_preempt_decide": (C.c_int, [P(split_queue_state), P(C.c_uint32)]),
         "split_qos_simulate": (C.c_int, [P(C.c_int64), P(C.c_uint32), C.c_uint32, C.c_uint32, P(C.c_uint32),
@@ -104,7 +111,7 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_eval_batch_host", "split_ga_run", "split_ga_population", "split_preempt_decide",
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
-            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain")
+            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain", "split_k_sweep")
 
 
 def lib():
@@ -261,6 +268,13 @@ class SplitGA:
             out = np.empty(n, dtype=np.float64)
         _check(_lib.split_eval_batch_host(self._h, _ptr(b), n, _ptr(out)), "split_eval_batch_host")
         return out
+
+    def k_sweep(self, k_lo: int, k_hi: int, generations: int, seed: int):
+        """f3: fixed-k GA per k in [k_lo, k_hi]; returns (k_best, [per-k dicts])."""
+        res = (split_k_result * (k_hi - k_lo + 1))()
+        kb = C.c_uint32(0)
+        _check(_lib.split_k_sweep(self._h, k_lo, k_hi, generations, seed, res, C.byref(kb)), "split_k_sweep")
+        return kb.value, [{f: getattr(r, f) for f, _ in split_k_result._fields_} for r in res]
 
     def set_chain(self, latencies_ns, cut_overhead_ns=None) -> None:
         """Replace the handle's chain (same n_ops): host arrays, uploaded on the handle's stream."""

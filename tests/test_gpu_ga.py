@@ -200,3 +200,31 @@ def test_set_chain_matches_fresh_handle(S):
     assert r["fitness"] == o["fitness"] and np.array_equal(r["bits"], o["bits"])
     assert np.array_equal(bits, o["population"][0])
     assert np.array_equal(_fbits(fit), _fbits(o["fitness_all"][0]))
+
+
+def test_k_sweep_eq1_choice(S):
+    """f3 (R21): split_k_sweep == one oracle fixed-k GA per k, and with a
+    constant per-cut overhead (S1 fixed per k) each k's best reaches the exact
+    minimum S2 of the DP, so the chosen k is the exact argmin of Eq. 1's wait
+    S2 / (2 S1) over k, computed here from the oracle DP."""
+    lat, ovh = wl.c1_chain(overhead="const")
+    delta = int(ovh[0])
+    with S.SplitGA(lat, ovh, pop_size=256, n_elite=4, k_min=2, k_max=12) as h:
+        kb, res = h.k_sweep(2, 12, 50, 42)
+        r_after = h.run(3, 1)                       # the handle's own k range is restored
+    o_after = oracle.ga_run(lat, ovh, 3, 1, pop_size=256, n_elite=4, k_min=2, k_max=12)
+    assert r_after["fitness"] == o_after["fitness"]
+    V = oracle.dp(lat, delta, 12)
+    T = int(lat.sum())
+    waits = {}
+    for r in res:
+        k = r["k"]
+        o = oracle.ga_run(lat, ovh, 50, 42, pop_size=256, n_elite=4, k_min=k, k_max=k)
+        assert r["fitness"] == o["fitness"] and r["var_num"] == o["var_num"]
+        assert r["expected_wait_ns"] == o["s2"] / (2.0 * o["s1"])
+        S1 = T + (k - 1) * delta
+        s2_min = (int(V[k]) + S1 * S1) // k
+        assert (int(V[k]) + S1 * S1) % k == 0
+        waits[k] = s2_min / (2.0 * S1)
+        assert r["expected_wait_ns"] == waits[k]
+    assert kb == min(waits, key=lambda k: (waits[k], k))
