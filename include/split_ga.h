@@ -60,8 +60,9 @@ typedef struct {
     double p_crossover;         /* [0,1]  one-point crossover probability    (P@21745-21902) */
     double p_mutation;          /* [0,1]  per-child one-bit-flip probability (P@21906-21963) */
     uint32_t k_min, k_max;      /* block-count range, 1 <= k_min <= k_max <= n_ops (R6)  */
-    uint32_t front_skip;        /* init draws cut positions from [front_skip, n_ops-2]
-                                   (observation "far from the front", P@19343-19437)     */
+    uint32_t front_skip;        /* every cut the GA places (init, mutation, repair) lies in
+                                   [front_skip, n_ops-2] (observation "far from the
+                                   front", P@19225-19437; R22)               */
     uint32_t stall_generations; /* stop after this many generations without a strictly
                                    better fitness; 0 = off               (P@22056-22160) */
     const int64_t* cut_overhead_ns; /* host, n_ops-1 entries: extra time the block after

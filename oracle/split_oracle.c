@@ -364,7 +364,7 @@ static uint32_t ga_tournament(const ga_ctx* g, uint32_t gid, uint32_t gen, const
     return best;
 }
 
-/* repair (R6): force popcount into [k_min-1, k_max-1] by uniform rank-select */
+/* repair (R17): force popcount into [k_min-1, k_max-1] by uniform rank-select */
 static void ga_repair(const ga_ctx* g, uint32_t gid, uint32_t gen, uint64_t* row)
 {
     uint32_t c = count_cuts(g, row);
@@ -376,9 +376,12 @@ static void ga_repair(const ga_ctx* g, uint32_t gid, uint32_t gen, uint64_t* row
             if (get_bit(row, pos)) { if (seen == r) { clr_bit(row, pos); break; } ++seen; }
         --c;
     }
+    /* cuts are added only in [front_skip, n-2] (R22: every operator keeps away from
+       the front, P@19225-19437); no individual ever has a cut below front_skip */
+    uint32_t f = g->p->front_skip;
     while (c < g->p->k_min - 1) {
-        uint32_t r = uniform_below(draw(g->seed, gid, gen, TAG_REPAIR, d++), npos - c);
-        for (uint32_t pos = 0, seen = 0; pos < npos; ++pos)
+        uint32_t r = uniform_below(draw(g->seed, gid, gen, TAG_REPAIR, d++), npos - f - c);
+        for (uint32_t pos = f, seen = 0; pos < npos; ++pos)
             if (!get_bit(row, pos)) { if (seen == r) { set_bit(row, pos); break; } ++seen; }
         ++c;
     }
@@ -524,7 +527,9 @@ int or_ga_run(uint32_t n, const int64_t* lat, const int64_t* ovh, const or_ga_pa
                     uint64_t* ch = P1 + (size_t)cs[h] * W;
                     uint32_t m0 = draw(seed, gidh, gen, TAG_MUTATE, 0);
                     uint32_t m1 = draw(seed, gidh, gen, TAG_MUTATE, 1);
-                    if ((uint64_t)m0 < thr_m) flip_bit(ch, uniform_below(m1, (uint64_t)(n - 1)));
+                    /* mutation flips a uniform position of [front_skip, n-2] (R22) */
+                    if ((uint64_t)m0 < thr_m)
+                        flip_bit(ch, p->front_skip + uniform_below(m1, (uint64_t)(n - 1 - p->front_skip)));
                     ga_repair(&g, gidh, gen, ch);
                     /* Step 2 — profile + fitness of the offspring (Eq. 2) */
                     F1[cs[h]] = or_fitness_value(n, lat, ovh, ch, p->k_min, p->k_max);

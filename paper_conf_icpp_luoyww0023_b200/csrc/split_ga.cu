@@ -74,9 +74,11 @@ __device__ __forceinline__ uint32_t select_bit(uint64_t m, uint32_t r)
     return pos;
 }
 
-// clear (set) the r-th set (unset) valid position, ascending order
+// clear (set) the r-th set (unset) valid position, ascending order; unset
+// positions below f (front_skip) are not candidates (R22)
 template <int WT>
-__device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch, uint32_t r, bool among_set)
+__device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch, uint32_t r, bool among_set,
+                                                uint32_t f)
 {
     // find the word holding the r-th candidate position, then toggle it with a mask
     uint32_t wi = 0xFFFFFFFFu, rr = 0;
@@ -84,7 +86,9 @@ __device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch
 #pragma unroll
     for (int i = 0; i < WT; ++i) {
         if (i < (int)ch.W) {
-            const uint64_t m = (among_set ? row.w[i] : ~row.w[i]) & word_mask(ch, i);
+            const uint32_t lo = 64u * i;
+            const uint64_t front = (f <= lo) ? ~0ull : (f >= lo + 64u ? 0ull : ~((1ull << (f - lo)) - 1ull));
+            const uint64_t m = (among_set ? row.w[i] : (~row.w[i] & front)) & word_mask(ch, i);
             const uint32_t c = __popcll(m);
             const bool here = (wi == 0xFFFFFFFFu) && r < c;
             wi = here ? (uint32_t)i : wi;
@@ -1016,11 +1020,11 @@ __device__ __forceinline__ void repair(const GaArgs& a, Row<WT>& row, uint32_t g
     Draws dr(gid, g, TAG_REPAIR, a.key0, a.key1);
     const uint32_t npos = ch.n - 1;
     while (c > ch.k_max - 1) {
-        row_toggle_rank(row, ch, below(dr.next(), c), true);
+        row_toggle_rank(row, ch, below(dr.next(), c), true, 0u);
         --c;
     }
-    while (c < ch.k_min - 1) {
-        row_toggle_rank(row, ch, below(dr.next(), npos - c), false);
+    while (c < ch.k_min - 1) {                  // cuts are added only in [front_skip, n-2] (R22)
+        row_toggle_rank(row, ch, below(dr.next(), npos - a.front_skip - c), false, a.front_skip);
         ++c;
     }
 }
@@ -1127,7 +1131,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
             }
         }
         if (tr) a.trace[(g - a.g_begin) * 16 + 13] = gtimer() + 0 * A.w[0];
-        if ((uint64_t)dr.mu.x < a.thr_m) row_xor_bit(A, below(dr.mu.y, ch.n - 1));      // a6
+        if ((uint64_t)dr.mu.x < a.thr_m)                                                   // a6 (R22)
+            row_xor_bit(A, a.front_skip + below(dr.mu.y, ch.n - 1 - a.front_skip));
         repair(a, A, gid, g);                                                              // a7
         if (tr) a.trace[(g - a.g_begin) * 16 + 10] = gtimer() + 0 * A.w[0];
         const double f = eval_regs(ch, sP, sO, A, nullptr, srow);                         // a2

@@ -88,6 +88,7 @@ def test_general_select_path_exercised(S):
     dict(pop_size=128, n_elite=8, p_crossover=0.0, p_mutation=0.0, k_min=1, k_max=105),
     dict(pop_size=128, n_elite=8, p_crossover=1.0, p_mutation=1.0),
     dict(pop_size=128, n_elite=8, k_min=5, k_max=5, front_skip=60),
+    dict(pop_size=256, n_elite=8, k_min=3, k_max=9, front_skip=90, p_mutation=1.0),
     dict(pop_size=128, n_elite=8, k_min=1, k_max=3),
 ])
 def test_edge_parameters(S, kw):

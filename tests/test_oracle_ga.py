@@ -159,3 +159,22 @@ def test_invalid_params_rejected():
         oracle.ga_run(lat, ovh, 1, 1, pop_size=256, n_elite=4, tournament_size=33)
     with pytest.raises(ValueError):
         oracle.ga_run(lat, ovh, 1, 1, pop_size=256, n_elite=4, k_min=5, k_max=4)
+
+
+def test_guided_operators_keep_the_front_clear():
+    # R22 (P@19225-19437): with front_skip = 200 every operator (init, mutation, the
+    # cuts repair adds) stays in [200, n-2]; high mutation and a wide k range make
+    # mutation and both repair directions fire many times
+    lat, ovh = wl.chain("bert_base")
+    n = len(lat)
+    r = oracle.ga_run(lat, ovh, 15, 3, pop_size=512, n_elite=8, k_min=3, k_max=6, front_skip=200,
+                      p_mutation=1.0, want_population=True)
+    pop = r["population"][0]
+    c = _popcount_rows(pop, n)
+    assert np.all((c >= 2) & (c <= 5))
+    assert np.all(pop[:, :3] == 0)
+    assert np.all(pop[:, 3] & np.uint64((1 << 8) - 1) == 0)
+    # front_skip = 0 leaves the operators as before: mutation reaches position 0..n-2
+    r0 = oracle.ga_run(lat, ovh, 15, 3, pop_size=512, n_elite=8, k_min=3, k_max=6, front_skip=0,
+                       p_mutation=1.0, want_population=True)
+    assert np.any(r0["population"][0][:, 0] != 0)
