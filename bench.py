@@ -206,6 +206,7 @@ def main():
     ap.add_argument("--no-exact", action="store_true")
     ap.add_argument("--no-ga-big", action="store_true")
     ap.add_argument("--no-qos", action="store_true")
+    ap.add_argument("--no-c3", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
@@ -460,6 +461,33 @@ def main():
                                       "paper-five chains in 4 GA-chosen blocks each",
                           "blocks_ms": [[round(b / 1e6, 3) for b in bl] for bl in qb], **qout}
         del da, dt
+
+    # C3 (BASELINE configs[2]): fixed-k GA for k = 2..32 on VGG-16 / MobileNetV2-shaped chains with a
+    # constant per-cut overhead, against the exact O(k n^2) DP optimum (f3 split_k_sweep drives the runs)
+    if not args.no_c3:
+        c3 = {}
+        for name in ("vgg16", "mobilenetv2"):
+            lc, _ = wl.chain(name)
+            oc, delta = wl.constant_overhead(lc)
+            kmax = min(32, len(lc))
+            with S.SplitGA(lc, oc, pop_size=65536, n_elite=1024, k_min=2, k_max=kmax, device=local,
+                           stream=stream) as hc:
+                s2 = hc.dp_min_s2(kmax)
+                t0c = time.perf_counter()
+                kb, res = hc.k_sweep(2, kmax, 200, 3)
+                tc = time.perf_counter() - t0c
+            T = int(lc.sum())
+            gaps, at_opt = [], 0
+            for r in res:
+                k = r["k"]
+                S1 = T + (k - 1) * delta
+                v_dp = k * int(s2[k]) - S1 * S1
+                gaps.append(r["var_num"] / v_dp - 1.0 if v_dp > 0 else float(r["var_num"] != 0))
+                at_opt += int(r["var_num"] == v_dp)
+            c3[name] = {"k_range": [2, kmax], "runs_at_dp_optimum": at_opt, "runs": len(res),
+                        "max_rel_excess_variance": max(gaps), "k_eq1_best": kb,
+                        "wall_s_all_k": tc, "generations_per_k": 200, "pop": 65536}
+        out["c3_k_sweep_vs_dp"] = c3
 
     # f1 exact solver: exhaustive enumeration of all 2^32 splits of a 33-op chain
     if not args.no_exact:
