@@ -289,7 +289,12 @@ def main():
                 "frac": achieved_gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
                 "traffic": _profile_traffic("ga_kernel_per_launch"),
                 "algorithmic_bytes_per_generation": gen_bytes,
-                "launch_ms_avg": loop_avg_ms, "share_of_step": loop_avg_ms / (t_max_ms / args.steps)}
+                "launch_ms_avg": loop_avg_ms, "share_of_step": loop_avg_ms / (t_max_ms / args.steps),
+                "note": ("C2's 1.7 MB working set is L2-resident (ncu DRAM traffic per 500-generation launch is "
+                         "the 'traffic' field): the kernel is bound by per-generation latency (two dependent L2 "
+                         "round trips, the fused eval and one grid barrier per generation), not by HBM; the same "
+                         "kernel's HBM regime is 'ga_hbm_regime', the HBM-bound K1 is 'eval_batch' "
+                         "(profiles/r01_notes.md)")}
 
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
