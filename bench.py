@@ -367,28 +367,34 @@ def main():
                          "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
                          "traffic": _profile_traffic("eval_batch_kernel_c5"),
                          "algorithmic_bytes_per_candidate": bpc}}
-        # C5 population sweep (BASELINE configs[4]: 1K-64M candidates): the 2^24 rows tiled on the device
+        # C5 population sweep (BASELINE configs[4]: 1K-64M candidates at 1/2/4/8 GPUs): each total size is
+        # sharded over the ranks (contiguous rows, no exchange), the 2^24 generated rows tiled on the device;
+        # time = max over ranks, value = all candidates / that time
         sweep = []
         for lg in (10, 14, 18, 22, 24, 26):
             n = 1 << lg
-            if n <= C5_EVAL_N:
-                b_n = bits[:n]
+            lo, hi = D.shard_range(n, rank, world)
+            n_loc = hi - lo
+            if n_loc <= C5_EVAL_N:
+                b_n = bits[:n_loc]
             else:
-                b_n = bits.repeat(n // C5_EVAL_N, 1)
-            f_n = torch.empty(n, dtype=torch.float64, device=dev)
-            h5.eval_batch(b_n, n, f_n)
+                b_n = bits.repeat((n_loc + C5_EVAL_N - 1) // C5_EVAL_N, 1)[:n_loc]
+            f_n = torch.empty(max(n_loc, 1), dtype=torch.float64, device=dev)
+            h5.eval_batch(b_n, n_loc, f_n)
             reps = 5 if lg >= 22 else 50
             z0, z1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            barrier()
             torch.cuda.synchronize()
             z0.record(stream)
             for _ in range(reps):
-                h5.eval_batch(b_n, n, f_n)
+                h5.eval_batch(b_n, n_loc, f_n)
             z1.record(stream)
             torch.cuda.synchronize()
-            zms = z0.elapsed_time(z1) / reps
+            zms, _, _ = D.reduce_max_sum(z0.elapsed_time(z1) / reps, 0.0, device=dev)
             zg = bpc * n / (zms / 1000.0) / 1e9
-            sweep.append({"n_cand": n, "ms": zms, "evals_per_s": n / (zms / 1000.0), "gbs": zg,
-                          "frac": zg / peaks["hbm_gbs"], "l2_resident": bpc * n < 100e6})
+            sweep.append({"n_cand": n, "n_gpus": world, "ms": zms, "evals_per_s": n / (zms / 1000.0), "gbs": zg,
+                          "frac_of_n_gpus_peak": zg / (peaks["hbm_gbs"] * world),
+                          "l2_resident": bpc * n_loc < 100e6})
             del b_n, f_n
         out["eval_batch"]["sweep"] = sweep
         h5.close()
