@@ -207,6 +207,7 @@ def main():
     ap.add_argument("--no-ga-big", action="store_true")
     ap.add_argument("--no-qos", action="store_true")
     ap.add_argument("--no-c3", action="store_true")
+    ap.add_argument("--no-c4", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
@@ -434,6 +435,37 @@ def main():
                          "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": bgbs / peaks["hbm_gbs"],
                          "peak_src": peaks["src"], "algorithmic_bytes_per_generation": gbytes,
                          "launch_ms_avg": bl}}
+
+    # C4 (BASELINE configs[3]): BERT-base chain, one island of 1,048,576 per GPU, top-64 migration over NCCL
+    # every 10 generations, 200 generations; with --gpus 8 this is the 8M-individual island model
+    if not args.no_c4:
+        latc, ovhc = wl.chain("bert_base")
+        c4kw = dict(pop_size=1 << 20, n_elite=1024, tournament_size=4, p_crossover=0.9, p_mutation=0.2,
+                    k_min=2, k_max=32)
+        c4isl = dict(**D.island_layout(rank, world, 1), migration_interval=MIGRATION_INTERVAL if world > 1 else 0,
+                     n_migrants=N_MIGRANTS if world > 1 else 0)
+        with S.SplitGA(latc, ovhc, device=local, stream=stream, comm=comm, **c4kw, **c4isl) as hc4:
+            hc4.run(20, 90)
+            c4ms, c4ev = [], 0
+            for i in range(3):
+                flush.fill_(i)
+                barrier()
+                torch.cuda.synchronize()
+                q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                q0.record(stream)
+                rc4 = hc4.run(200, 91 + i)
+                q1.record(stream)
+                torch.cuda.synchronize()
+                c4ms.append(q0.elapsed_time(q1))
+                c4ev += rc4["evaluations"]
+        t4, ev4, _ = D.reduce_max_sum(sum(c4ms), float(c4ev), device=dev)
+        out["c4_island_model"] = {
+            "workload": f"C4: bert_base chain (n=400, W=7), one island of 1,048,576 per GPU ({world} islands), "
+                        "E=1024, s=4, 200 generations per step" +
+                        (f", top-{N_MIGRANTS} migrants over NCCL every {MIGRATION_INTERVAL} generations" if world > 1
+                         else ", no migration (1 island)"),
+            "evals_per_s": ev4 / (t4 / 1000.0), "ms_per_step": t4 / len(c4ms),
+            "gens_per_s": 200 / ((t4 / len(c4ms)) / 1000.0), "n_gpus": world, "scaling": "weak"}
 
     # f2 QoS simulator: Table 2's heaviest scenario (lambda = 110 ms, 1000 requests) over the
     # paper-five chains split into 4 blocks by the GA, Algorithm 1 vs FIFO, 65,536 replicas
