@@ -1019,9 +1019,33 @@ __device__ __forceinline__ void repair(const GaArgs& a, Row<WT>& row, uint32_t g
     if (c + 1 >= ch.k_min && c + 1 <= ch.k_max) return;
     Draws dr(gid, g, TAG_REPAIR, a.key0, a.key1);
     const uint32_t npos = ch.n - 1;
-    while (c > ch.k_max - 1) {
-        row_toggle_rank(row, ch, below(dr.next(), c), true, 0u);
-        --c;
+    if (c > ch.k_max - 1) {
+        // removals: per-word cut counts computed once, then each step finds its word by
+        // a running prefix (no POPC) and clears the rr-th set bit of that word
+        uint32_t cw[WT];
+#pragma unroll
+        for (int i = 0; i < WT; ++i) cw[i] = (i < (int)ch.W) ? (uint32_t)__popcll(row.w[i] & word_mask(ch, i)) : 0u;
+        while (c > ch.k_max - 1) {
+            uint32_t r = below(dr.next(), c);
+            uint32_t wi = 0xFFFFFFFFu, rr = 0;
+            uint64_t mw = 0;
+#pragma unroll
+            for (int i = 0; i < WT; ++i) {
+                const bool here = (wi == 0xFFFFFFFFu) && r < cw[i];
+                wi = here ? (uint32_t)i : wi;
+                mw = here ? (row.w[i] & word_mask(ch, i)) : mw;
+                rr = here ? r : rr;
+                r -= (wi == 0xFFFFFFFFu) ? cw[i] : 0u;
+            }
+            const uint64_t bit = 1ull << select_bit(mw, rr);
+#pragma unroll
+            for (int i = 0; i < WT; ++i) {
+                const bool me = (uint32_t)i == wi;
+                row.w[i] ^= me ? bit : 0ull;
+                cw[i] -= me ? 1u : 0u;
+            }
+            --c;
+        }
     }
     while (c < ch.k_min - 1) {                  // cuts are added only in [front_skip, n-2] (R22)
         row_toggle_rank(row, ch, below(dr.next(), npos - a.front_skip - c), false, a.front_skip);
