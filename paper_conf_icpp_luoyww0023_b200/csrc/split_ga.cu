@@ -1123,6 +1123,8 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
     const uint32_t chunks = (nchild + 31u) / 32u;
     const uint32_t first = warp * a.cpi + wl;
     const uint64_t tau = __ldcg(tau_ptr);     // lagged elite threshold: stable during this phase
+    ChildDraws nxt_dr;
+    bool have_next = false;
     for (uint32_t cidx_ = first; cidx_ < chunks; cidx_ += nwarps * a.cpi) {
         const uint32_t base = cidx_ * 32u;
         const uint32_t t = base + lane;
@@ -1134,6 +1136,7 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
                         g - a.g_begin < a.trace_gens && cidx_ == wl;
         ChildDraws dr;
         if (cidx_ == first && have_pre) dr = pre;
+        else if (WT >= 8 && have_next) dr = nxt_dr;
         else dr = child_draws(a, gid, h, g);
         const uint32_t mine =
             valid ? tournament<WT>(a, gid, g, fitc, dr.sel, (cidx_ == first && have_pre) ? fpre : nullptr) : 0u;   // a4
@@ -1144,6 +1147,16 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         Row<WT> A, B;
         row_load(A, popc + (size_t)mine * W, W);
         row_load(B, popc + (size_t)other * W, W);
+        // wide rows (several chunks per warp at large N): the next chunk's Philox draws,
+        // computed while this chunk's parent rows are in flight
+        if constexpr (WT >= 8) {
+            const uint32_t cn = cidx_ + nwarps * a.cpi;
+            have_next = cn < chunks;
+            if (have_next) {
+                const uint32_t tn = cn * 32u + lane;
+                nxt_dr = child_draws(a, (a.island_base + i) * N + E + tn, tn & 1u, g);
+            }
+        }
         if (tr) a.trace[(g - a.g_begin) * 16 + 9] = gtimer() + 0 * (A.w[0] ^ B.w[0]);
         if ((uint64_t)dr.xo.x < a.thr_c && ch.n >= 3) {                                   // a5
             const uint32_t x = 1 + below(dr.xo.y, ch.n - 2);
