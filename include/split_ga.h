@@ -200,7 +200,8 @@ void split_comm_destroy(void* comm);
 int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* min_v_per_k, uint64_t* argmin_per_k);
 
 /* a0 again on a live handle: replace its chain (same n_ops) -- new per-operator
- * latencies and cut overheads (host, copied; NULL overheads = 0), validated and
+ * latencies (profiled per operator, P@18308-18385) and cut overheads (the data
+ * transmission a cut adds, P@13239-13520; host, copied; NULL = 0), validated and
  * guarded exactly as split_ga_create does for the handle's k_max -- and upload
  * the tables stream-ordered on the handle's stream.  No allocation: the serving
  * path re-splits a model whose profile changed without create/destroy.  The
