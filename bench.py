@@ -163,6 +163,33 @@ def cpu_baseline_oracle(generations: int) -> dict:
             "gens_per_s": generations / dt}
 
 
+def _oracle_eval_shard(args):
+    import oracle
+    from paper_conf_icpp_luoyww0023_b200 import workloads as wl
+    n_cand, seed = args
+    lat, ovh = wl.chain("synthetic_1024")
+    pop = wl.uniform_k_population_fast(len(lat), n_cand, seed=seed)
+    t0 = time.perf_counter()
+    oracle.fitness_batch(lat, ovh, pop, 2, 32)
+    return time.perf_counter() - t0
+
+
+def cpu_eval_all_cores(n_per_core: int = 1 << 18) -> dict:
+    """The oracle's fitness (plain C, single-threaded) as P independent processes on disjoint
+    shards of C5 candidates, P = the host cores this process may use."""
+    import multiprocessing as mp
+    P = len(os.sched_getaffinity(0))
+    ctx = mp.get_context("spawn")
+    with ctx.Pool(P) as pool:
+        ts = pool.map(_oracle_eval_shard, [(n_per_core, 1000 + i) for i in range(P)])
+    wall = max(ts)                                   # oracle time of the slowest process
+    cpu = open("/proc/cpuinfo").read().split("model name")[1].split("\n")[0].strip(": \t") \
+        if os.path.exists("/proc/cpuinfo") and "model name" in open("/proc/cpuinfo").read() else "unknown"
+    return {"value": P * n_per_core / wall, "unit": UNIT, "cores": P, "kind": "oracle",
+            "sample": f"oracle fitness (C5 rows, n = 1024) in {P} processes x {n_per_core} candidates; "
+                      f"slowest process {wall:.2f} s of oracle time", "cpu": cpu}
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -552,6 +579,10 @@ def main():
     out["clocks"] = clk.summary()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline_oracle(CPU_SAMPLE_GENERATIONS)
+        try:
+            out["cpu_baseline"]["eval_all_cores"] = cpu_eval_all_cores()
+        except Exception as e:                      # reported baseline only; never fails the run
+            out["cpu_baseline"]["eval_all_cores"] = {"unavailable": repr(e)[:200]}
     out["paper_context"] = ("PAPER.md profiles 'over 20,000 candidates' offline on a Jetson Nano at ~1 s per "
                             "candidate (287,980 candidates > 80 h, P@9901-10019): ~1 eval/s; context only")
     h.close()
