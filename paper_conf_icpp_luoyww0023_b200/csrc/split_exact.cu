@@ -108,8 +108,11 @@ __global__ void __launch_bounds__(kExhThreads) exh_kernel(ExhArgs a)
     constexpr uint32_t NW = kExhThreads / 32;
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t nb = 1u << a.c, rows = a.m - a.c + 1;
-    ExhEntry* s_tab = (ExhEntry*)smem;                                    // [rows][nb]
-    uint32_t* s_A = (uint32_t*)(s_tab + rows * nb);                       // [m+1]
+    // [rows][nb + 1]: one pad entry per row shifts each row by 4 banks, so lanes at
+    // different lowest high cuts H (different rows, same bl) read different banks
+    const uint32_t pitch = nb + 1;
+    ExhEntry* s_tab = (ExhEntry*)smem;
+    uint32_t* s_A = (uint32_t*)(s_tab + rows * pitch);                    // [m+1]
     uint32_t* s_B = s_A + ((a.m + 1 + 3) & ~3u);                          // [m]
     ExhThr* s_thr = (ExhThr*)(s_B + ((a.m + 3) & ~3u));                   // [65]
     uint64_t* s_kv = (uint64_t*)(s_thr + 65);                             // [65] MINV / ARGMIN
@@ -120,7 +123,7 @@ __global__ void __launch_bounds__(kExhThreads) exh_kernel(ExhArgs a)
     ExhResult* s_red = (ExhResult*)(s_qk + NW * kExhQ);                   // [NW]
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
 
-    for (uint32_t i = tid; i < rows * nb; i += blockDim.x) s_tab[i] = ((const ExhEntry*)a.tab)[i];
+    for (uint32_t i = tid; i < rows * nb; i += blockDim.x) s_tab[(i / nb) * pitch + i % nb] = ((const ExhEntry*)a.tab)[i];
     for (uint32_t i = tid; i <= a.m; i += blockDim.x) s_A[i] = a.A[i];
     for (uint32_t i = tid; i < a.m; i += blockDim.x) s_B[i] = a.B[i];
     for (uint32_t k = tid; k < 65; k += blockDim.x) {
@@ -194,7 +197,7 @@ __global__ void __launch_bounds__(kExhThreads) exh_kernel(ExhArgs a)
     const uint32_t c = a.c;
     for (uint64_t s = s0; __any_sync(0xFFFFFFFFu, active && s < s1); ++s) {
         const bool live = active && s < s1;
-        const ExhEntry* row = s_tab + (size_t)(H - c) * nb;
+        const ExhEntry* row = s_tab + (size_t)(H - c) * pitch;
         const uint32_t kb = ku + 1;
         const uint32_t S1b = T + OVu;
         for (uint32_t bl = 0; bl < nb; ++bl) {
@@ -356,7 +359,7 @@ __global__ void __launch_bounds__(1024) dp_kernel(const uint32_t* P /*[n+1]*/, c
 size_t exh_smem_bytes(const ExhArgs& a)
 {
     const size_t rows = a.m - a.c + 1, nb = 1u << a.c, NW = kExhThreads / 32;
-    return rows * nb * sizeof(ExhEntry) + 4 * (((a.m + 1 + 3) & ~3u) + ((a.m + 3) & ~3u)) + 65 * sizeof(ExhThr) +
+    return rows * (nb + 1) * sizeof(ExhEntry) + 4 * (((a.m + 1 + 3) & ~3u) + ((a.m + 3) & ~3u)) + 65 * sizeof(ExhThr) +
            65 * 8 + NW * kExhQ * (8 + 8 + 4 + 4) + NW * sizeof(ExhResult);
 }
 
