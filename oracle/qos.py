@@ -22,6 +22,15 @@ pinned event semantics are DESIGN.md reading R20:
   has started leaves Q; its end-to-end latency t_ete = end of its last block
   minus its arrival.
 
+f4 elastic splitting (ELASTIC, reading R23; §3.3 P@22612-23675:
+splitting "is temporarily disabled" under "particularly high request density"
+and "temporarily suspended" when "an excessive number of requests of the same
+type are present"; the paper gives no thresholds, so they are parameters):
+a request of type m arriving when Q holds >= d_max entries, or >= s_max
+entries of type m, runs unsplit -- one block of unsplit[m] -- and is appended
+at the tail of Q (no preemption); otherwise it is split and placed by
+Algorithm 1 as under ALG1.  An unsplit entry in Q has Ext_left = unsplit[m].
+
 Statistics (request order i = 0..n-1): violations per alpha = #{i : 1000 t_ete
 > alpha_milli Ext}; rr_sum = sum of RN(t_ete/Ext) added in order, rr_sq = sum of
 RN(RR*RR) added in order (IEEE doubles, as the CUDA path adds them).
@@ -32,7 +41,7 @@ from dataclasses import dataclass
 
 from oracle.preempt import Request, preemption
 
-FIFO, ALG1 = 0, 1
+FIFO, ALG1, ELASTIC = 0, 1, 2
 
 
 @dataclass
@@ -40,10 +49,12 @@ class _Entry:
     req: int
     ext_left: int
     blk: int
+    unsplit: bool = False
 
 
-def simulate(blocks: list[list[int]], arrival: list[int], types: list[int], policy: int) -> list[int]:
-    """Return t_ete (ns) of every request."""
+def simulate(blocks: list[list[int]], arrival: list[int], types: list[int], policy: int,
+             unsplit: list[int] | None = None, d_max: int = 0, s_max: int = 0) -> list[int]:
+    """Return t_ete (ns) of every request.  unsplit, d_max, s_max: ELASTIC only."""
     n = len(arrival)
     ext = [sum(b) for b in blocks]
     t_ete = [None] * n
@@ -59,7 +70,7 @@ def simulate(blocks: list[list[int]], arrival: list[int], types: list[int], poli
         if busy_until is not None or not Q:
             return
         h = Q[0]
-        b = blocks[types[h.req]][h.blk]
+        b = unsplit[types[h.req]] if h.unsplit else blocks[types[h.req]][h.blk]
         busy_until = now + b
         running = h.req
         h.blk += 1
@@ -80,12 +91,17 @@ def simulate(blocks: list[list[int]], arrival: list[int], types: list[int], poli
         else:
             now = arrival[i]                           # arrival (first on ties)
             m = types[i]
+            entry = _Entry(i, ext[m], 0)
+            same = sum(1 for e in Q if types[e.req] == m)
             if policy == FIFO:
+                pos = len(Q)
+            elif policy == ELASTIC and (len(Q) >= d_max or same >= s_max):
+                entry = _Entry(i, unsplit[m], 0, True)         # splitting suspended (R23)
                 pos = len(Q)
             else:
                 queue = [Request(types[e.req], arrival[e.req], ext[types[e.req]], e.ext_left) for e in Q]
                 pos = preemption(now, 1.0, queue, Request(m, now, ext[m], ext[m]))
-            Q.insert(pos, _Entry(i, ext[m], 0))
+            Q.insert(pos, entry)
             i += 1
             dispatch(now)
     return t_ete

@@ -73,3 +73,51 @@ def test_same_type_never_passes_and_busy_periods_are_policy_free():
         # one type only: Algorithm 1 never reorders (line 6) -> identical to FIFO
         same = [0] * len(a)
         assert qos.simulate(blocks, a, same, qos.ALG1) == qos.simulate(blocks, a, same, qos.FIFO)
+
+
+# ---- f4 elastic splitting (ELASTIC, R23; §3.3 P@22612-23675) ----
+
+def test_elastic_worked_examples_by_hand():
+    # L: 3 blocks of 5 (Ext 15), unsplit T = 13 (no cut overheads); S: one block of 2 (T = 2)
+    blocks, uns = [[5, 5, 5], [2]], [13, 2]
+    big = 1 << 30
+    # density: S arrives to 1 pending request (L, blocks 2 and 3 not started).
+    # d_max = 1 -> splitting off for S: unsplit, at the tail, runs after L (15..17)
+    assert qos.simulate(blocks, [0, 1], [0, 1], qos.ELASTIC, uns, 1, big) == [15, 16]
+    # d_max = 2 -> S is split and passes L (Algorithm 1), as under ALG1
+    assert qos.simulate(blocks, [0, 1], [0, 1], qos.ELASTIC, uns, 2, big) == [17, 6]
+    # same type: a second L arrives while L is pending.  s_max = 1 -> it runs unsplit
+    # (13 ns, no overheads) after L: 15..28; s_max = 2 -> split, 15..30
+    assert qos.simulate(blocks, [0, 1], [0, 0], qos.ELASTIC, uns, big, 1) == [15, 27]
+    assert qos.simulate(blocks, [0, 1], [0, 0], qos.ELASTIC, uns, big, 2) == [15, 29]
+    # a queued unsplit request is passed by a later split arrival like any other:
+    # Q = [L (left 10), L' (unsplit 13)]; S at 2: 13*15 > 4 and 10*15 > 4 -> head;
+    # S runs at L's first block boundary 5..7, L 7..17, L' 17..30
+    assert qos.simulate(blocks, [0, 1, 2], [0, 0, 1], qos.ELASTIC, uns, big, 1) == [17, 29, 5]
+
+
+def test_elastic_thresholds_zero_is_fifo_lindley_of_unsplit_models():
+    # d_max = 0: splitting always off -> a FIFO single-server queue whose service
+    # time is the unsplit T of each request: end_i = max(a_i, end_{i-1}) + T(m_i)
+    arr, ty = wl.qos_requests(2, 300, 6_000_000, 3, seed=11)
+    blocks = wl.random_blocks(3, seed=4, k_hi=5, lo=500_000, hi=4_000_000)
+    uns = [sum(b) - 300_000 for b in blocks]
+    for r in range(2):
+        a = [int(x) for x in arr[r]]
+        t = [int(x) for x in ty[r]]
+        for d, s in ((0, 1 << 30), (1 << 30, 0)):
+            got = qos.simulate(blocks, a, t, qos.ELASTIC, uns, d, s)
+            end = 0
+            for i in range(len(a)):
+                end = max(a[i], end) + uns[t[i]]
+                assert got[i] == end - a[i]
+
+
+def test_elastic_infinite_thresholds_is_algorithm1():
+    arr, ty = wl.qos_requests(2, 200, 8_000_000, 4, seed=12)
+    blocks = wl.random_blocks(4, seed=5, k_hi=5, lo=500_000, hi=6_000_000)
+    uns = [sum(b) for b in blocks]
+    for r in range(2):
+        a = [int(x) for x in arr[r]]
+        t = [int(x) for x in ty[r]]
+        assert qos.simulate(blocks, a, t, qos.ELASTIC, uns, 1 << 30, 1 << 30) == qos.simulate(blocks, a, t, qos.ALG1)
