@@ -37,6 +37,7 @@ MIGRATION_INTERVAL, N_MIGRANTS = 10, 64
 C5_EVAL_N = 1 << 24           # split_eval_batch sub-measurement (C5: n = 1024, 2.3 GB of bitsets > L2)
 EXACT_N = 33                  # f1 sub-measurement: split_exhaustive over 2^32 splits
 QOS_REPLICAS = 65536          # f2 sub-measurement
+QOS_ELASTIC_D, QOS_ELASTIC_S = 3, 2   # f4: pending-request density / same-type thresholds (R23; the paper gives none)
 GA_BIG = dict(chain="bert_base", pop_size=1 << 22, n_elite=1024, tournament_size=4, p_crossover=0.9,
               p_mutation=0.2, k_min=2, k_max=32, generations=50)   # C4-shaped island of 4M: HBM regime
 CPU_SAMPLE_GENERATIONS = 100  # oracle cpu_baseline: about 10 s of one core
@@ -497,9 +498,10 @@ def main():
     # f2 QoS simulator: Table 2's heaviest scenario (lambda = 110 ms, 1000 requests) over the
     # paper-five chains split into 4 blocks by the GA, Algorithm 1 vs FIFO, 65,536 replicas
     if not args.no_qos:
-        qb = []
+        qb, quns = [], []
         for name in ("yolov2", "googlenet", "resnet50_122", "vgg19", "gpt2"):
             lq, oq = wl.chain(name)
+            quns.append(int(np.asarray(lq, dtype=np.int64).sum()))    # unsplit: T, no cut overheads
             with S.SplitGA(lq, oq, pop_size=4096, n_elite=64, k_min=4, k_max=4, device=local, stream=stream) as hq:
                 rq = hq.run(50, 1)
             qb.append(S.block_times(lq, oq, rq["bits"]))
@@ -508,14 +510,16 @@ def main():
         dt = torch.from_numpy(np.ascontiguousarray(typ.T)).to(dev)
         alphas = [1000 * a for a in range(2, 21)]
         qout = {}
-        for pol, pname in ((1, "algorithm1"), (0, "fifo")):
-            S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream)
+        # f4 elastic splitting (R23): thresholds are ours (the paper gives none, P@22612-23675)
+        el = {"unsplit": quns, "d_max": QOS_ELASTIC_D, "s_max": QOS_ELASTIC_S}
+        for pol, pname, kw in ((1, "algorithm1", {}), (0, "fifo", {}), (2, "elastic", el)):
+            S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream, **kw)
             torch.cuda.synchronize()
             qmss = []
             for _ in range(3):
                 q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 q0.record(stream)
-                te, viol, rr = S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream)
+                te, viol, rr = S.split_qos_simulate(qb, da, dt, alphas, pol, device=local, stream=stream, **kw)
                 q1.record(stream)
                 torch.cuda.synchronize()
                 qmss.append(q0.elapsed_time(q1))
@@ -527,6 +531,8 @@ def main():
             qout[pname] = {"requests_per_s": QOS_REPLICAS * 1000 / (qms / 1000.0), "ms": qms,
                            "violation_rate": {f"alpha={a // 1000}": float(x) for a, x in zip(alphas, v)},
                            "rr_mean": float(mean), "rr_std": sd}
+            if pol == 2:
+                qout[pname]["thresholds"] = {"d_max": QOS_ELASTIC_D, "s_max": QOS_ELASTIC_S}
         out["qos_sim"] = {"workload": f"f2: {QOS_REPLICAS} replicas x 1000 Poisson requests (lambda = 110 ms), "
                                       "paper-five chains in 4 GA-chosen blocks each",
                           "blocks_ms": [[round(b / 1e6, 3) for b in bl] for bl in qb], **qout}

@@ -177,6 +177,28 @@ int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint3
                        const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,
                        uint32_t* viol_out, double* rr_out, int device, void* stream);
 
+/* f4 — elastic model splitting (§3.3 P@22612-23675:
+ * "under conditions of particularly high request density, model splitting is
+ * temporarily disabled ... when an excessive number of requests of the same
+ * type are present, splitting is also temporarily suspended").  The paper
+ * gives no thresholds, so they are arguments (reading R23): a
+ * request of type m arriving when the pending queue holds >= d_max requests,
+ * or >= s_max requests of type m, runs UNSPLIT — one block of unsplit_ns[m]
+ * (the model without cut overheads, T) — and joins the queue tail (no
+ * preemption); otherwise it is split and placed by Algorithm 1 exactly as
+ * split_qos_simulate policy 1.  Queued unsplit requests take part in later
+ * Algorithm 1 scans with Ext_left = unsplit_ns[m].  Violations and response
+ * ratios use the same per-type Ext (sum of the split blocks) as
+ * split_qos_simulate, so the two are directly comparable; d_max = s_max =
+ * UINT32_MAX reproduces policy 1, d_max = 0 a FIFO queue of unsplit models.
+ *   unsplit_ns  host, n_types entries in [1, 2^32)
+ * Other arguments, layouts, synchronisation and errors: split_qos_simulate. */
+int split_qos_simulate_elastic(const int64_t* blocks_ns, const uint32_t* n_blocks, const int64_t* unsplit_ns,
+                               uint32_t n_types, uint32_t d_max, uint32_t s_max, const uint32_t* alpha_milli,
+                               uint32_t n_alpha, uint64_t n_rep, uint32_t n_req, const int64_t* arrival_ns,
+                               const uint32_t* type_id, int64_t* t_ete_out, uint32_t* viol_out, double* rr_out,
+                               int device, void* stream);
+
 /* Island communicator over NCCL (the libnccl.so.2 already loaded in the
  * process, e.g. by torch).  Rank r of `world` runs islands_per_device islands
  * starting at island_id = r*islands_per_device.  unique_id: 128 bytes from

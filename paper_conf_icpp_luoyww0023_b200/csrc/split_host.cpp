@@ -1115,14 +1115,23 @@ extern "C" int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out)
 // ------------------------------------------------------------------------
 // f2: QoS simulator (split_qos.cu)
 // ------------------------------------------------------------------------
-extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
-                                  const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep, uint32_t n_req,
-                                  const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,
-                                  uint32_t* viol_out, double* rr_out, int device, void* stream)
+static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
+                        const int64_t* unsplit_ns, uint32_t d_max, uint32_t s_max, const uint32_t* alpha_milli,
+                        uint32_t n_alpha, uint64_t n_rep, uint32_t n_req, const int64_t* arrival_ns,
+                        const uint32_t* type_id, int64_t* t_ete_out, uint32_t* viol_out, double* rr_out, int device,
+                        void* stream)
 {
     if (!blocks_ns || !n_blocks || n_types == 0 || n_types > 65535)
         return fail(SPLIT_E_INVAL, "split_qos_simulate: need 1..65535 model types with their blocks");
-    if (policy > 1) return fail(SPLIT_E_INVAL, "split_qos_simulate: policy must be 0 (FIFO) or 1 (Algorithm 1)");
+    if (policy > 2 || (policy == 2) != (unsplit_ns != nullptr))
+        return fail(SPLIT_E_INVAL, "split_qos_simulate: policy must be 0 (FIFO) or 1 (Algorithm 1); elastic needs unsplit_ns");
+    std::vector<uint32_t> uns;
+    if (policy == 2)
+        for (uint32_t m = 0; m < n_types; ++m) {
+            if (unsplit_ns[m] < 1 || unsplit_ns[m] >= ((int64_t)1 << 32))
+                return fail(SPLIT_E_RANGE, "split_qos_simulate_elastic: unsplit time out of [1, 2^32)");
+            uns.push_back((uint32_t)unsplit_ns[m]);
+        }
     if (n_alpha > kQosMaxAlpha || (n_alpha && !alpha_milli))
         return fail(SPLIT_E_INVAL, "split_qos_simulate: at most %u alpha thresholds", kQosMaxAlpha);
     if (n_rep == 0 || n_req == 0) return SPLIT_OK;
@@ -1152,6 +1161,7 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
     tab.insert(tab.end(), ext.begin(), ext.end());
     tab.insert(tab.end(), alpha_milli, alpha_milli + n_alpha);
     tab.insert(tab.end(), blk.begin(), blk.end());
+    tab.insert(tab.end(), uns.begin(), uns.end());
     tab.push_back(0);                                   // error flag
     QosArgs a;
     memset(&a, 0, sizeof(a));
@@ -1166,6 +1176,8 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
     a.t_ete = t_ete_out;
     a.viol = viol_out;
     a.rr = rr_out;
+    a.d_max = d_max;
+    a.s_max = s_max;
     if (qos_smem_bytes(a) > 227 * 1024) return fail(SPLIT_E_INVAL, "split_qos_simulate: model tables too large");
     // stream-ordered scratch (no device-wide synchronisation in cudaFree)
     uint32_t* d_tab = nullptr;
@@ -1180,6 +1192,7 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
     a.ext = d_tab + n_types + 1;
     a.alpha_milli = a.ext + n_types;
     a.blk_ns = a.alpha_milli + n_alpha;
+    a.uns = a.blk_ns + blk.size();
     a.err = d_tab + tab.size() - 1;
     CU(launch_qos(a, st));
     uint32_t err = 0;
@@ -1188,4 +1201,26 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
     if (err == 1) return fail(SPLIT_E_RANGE, "split_qos_simulate: arrivals not non-decreasing / negative, or type id >= n_types");
     if (err == 2) return fail(SPLIT_E_RANGE, "split_qos_simulate: more than %u pending requests (overloaded)", kQosQueue);
     return SPLIT_OK;
+}
+
+extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
+                                  const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep, uint32_t n_req,
+                                  const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,
+                                  uint32_t* viol_out, double* rr_out, int device, void* stream)
+{
+    if (policy > 1) return fail(SPLIT_E_INVAL, "split_qos_simulate: policy must be 0 (FIFO) or 1 (Algorithm 1)");
+    return qos_simulate(blocks_ns, n_blocks, n_types, policy, nullptr, 0, 0, alpha_milli, n_alpha, n_rep, n_req,
+                        arrival_ns, type_id, t_ete_out, viol_out, rr_out, device, stream);
+}
+
+extern "C" int split_qos_simulate_elastic(const int64_t* blocks_ns, const uint32_t* n_blocks, const int64_t* unsplit_ns,
+                                          uint32_t n_types, uint32_t d_max, uint32_t s_max,
+                                          const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep,
+                                          uint32_t n_req, const int64_t* arrival_ns, const uint32_t* type_id,
+                                          int64_t* t_ete_out, uint32_t* viol_out, double* rr_out, int device,
+                                          void* stream)
+{
+    if (!unsplit_ns) return fail(SPLIT_E_INVAL, "split_qos_simulate_elastic: NULL unsplit_ns");
+    return qos_simulate(blocks_ns, n_blocks, n_types, 2, unsplit_ns, d_max, s_max, alpha_milli, n_alpha, n_rep, n_req,
+                        arrival_ns, type_id, t_ete_out, viol_out, rr_out, device, stream);
 }

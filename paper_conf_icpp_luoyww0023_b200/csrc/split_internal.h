@@ -114,6 +114,7 @@ int exh_blocks_per_sm(const ExhArgs& a);
 constexpr uint32_t kQosThreads = 64;    // replicas per CTA (one per thread): 7 CTAs per SM fit 65,536 replicas in one wave
 constexpr uint32_t kQosQueue = 32;      // pending requests a replica may hold
 constexpr uint32_t kQosMaxAlpha = 32;
+constexpr uint32_t kQosUnsplit = 0xFFFFu; // block field of a queue entry that runs unsplit (f4)
 struct QosArgs {
     uint32_t n_types, n_blocks_total, n_alpha, policy;
     const uint32_t* blk_off;       // [n_types + 1] prefix of blocks per type
@@ -128,6 +129,10 @@ struct QosArgs {
     uint32_t* viol;                // [n_rep][n_alpha]
     double* rr;                    // [n_rep][2]
     uint32_t* err;                 // 0 ok, 1 bad arrival/type, 2 queue overflow
+    // f4 elastic splitting (policy 2, R23): a request arriving to >= d_max pending requests, or to >= s_max pending
+    // requests of its own type, runs unsplit (one block of uns[type] ns) and joins the tail
+    uint32_t d_max, s_max;
+    const uint32_t* uns;           // [n_types] unsplit latency T per type (policy 2 only)
 };
 size_t qos_smem_bytes(const QosArgs& a);
 cudaError_t launch_qos(const QosArgs& a, cudaStream_t st);

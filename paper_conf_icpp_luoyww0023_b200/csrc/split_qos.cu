@@ -31,10 +31,13 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     uint32_t* q_left = q_req + kQosQueue * kQosThreads;   // Ext_left (ns)
     uint32_t* q_tb = q_left + kQosQueue * kQosThreads;    // type | next block << 16
     uint32_t* s_viol = q_tb + kQosQueue * kQosThreads;    // [n_alpha][kQosThreads]
+    uint32_t* s_uns = s_viol + a.n_alpha * kQosThreads;   // [M] unsplit T (policy 2)
     for (uint32_t j = threadIdx.x; j <= a.n_types; j += blockDim.x) s_off[j] = a.blk_off[j];
     for (uint32_t j = threadIdx.x; j < a.n_types; j += blockDim.x) s_ext[j] = a.ext[j];
     for (uint32_t j = threadIdx.x; j < a.n_alpha; j += blockDim.x) s_alpha[j] = a.alpha_milli[j];
     for (uint32_t j = threadIdx.x; j < nb; j += blockDim.x) s_blk[j] = a.blk_ns[j];
+    if (a.policy == 2u)
+        for (uint32_t j = threadIdx.x; j < a.n_types; j += blockDim.x) s_uns[j] = a.uns[j];
     __syncthreads();
     const uint32_t tid = threadIdx.x;
     const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + tid;
@@ -53,11 +56,15 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     uint32_t next_t = n_req ? __ldcs(ty) : 0;
     int64_t prev_a = 0;
     uint32_t err = 0;
+    // lanes of this warp that hold a replica (the grid's last warp may be partial)
+    const uint64_t wbase = r - (tid & 31u);
+    const uint64_t nl = a.n_rep - wbase;
+    const unsigned wmask = nl >= 32 ? 0xFFFFFFFFu : ((1u << nl) - 1u);
     // start the next block of the queue head (executor idle)
     auto dispatch = [&]() {
         if (!idle || n == 0) return;
         const uint32_t tb = Q(q_tb, 0), m = tb & 0xFFFFu, blk = tb >> 16;
-        const uint32_t b = s_blk[s_off[m] + blk];
+        const uint32_t b = (blk == kQosUnsplit) ? s_uns[m] : s_blk[s_off[m] + blk];
         const uint32_t left = Q(q_left, 0) - b;
         run_req = Q(q_req, 0);
         run_arr = __ldg(arr + run_req * st);
@@ -76,48 +83,68 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
             Q(q_tb, 0) = tb + (1u << 16);
         }
     };
-    while (done < n_req) {
-        if (!idle && (i >= n_req || busy < next_a)) {
-            now = busy;                                   // block end
-            if (run_last) {
-                __stcs(te + run_req * st, now - run_arr);
-                ++done;
-            }
-            idle = true;
-            dispatch();
-        } else {
-            now = next_a;                                 // arrival (first on ties)
-            if (now < prev_a || now < 0 || next_t >= a.n_types) { err = 1u; break; }
-            prev_a = now;
-            const uint32_t m = next_t, e = s_ext[m];
-            uint32_t pos = n;
-            if (a.policy == 1u) {
-                // Algorithm 1 (R12): scan from the tail; stay behind the first request of
-                // the same type or with Ext_left * Ext <= Ext_left(new) * Ext(new)
-                const uint64_t key = (uint64_t)e * e;
-                pos = 0;
-                for (uint32_t j = n; j-- > 0;) {
-                    const uint32_t tj = Q(q_tb, j) & 0xFFFFu;
-                    if (tj == m || (uint64_t)Q(q_left, j) * s_ext[tj] <= key) { pos = j + 1; break; }
+    // One event per thread per warp-iteration, with the warp re-converged after each: the replicas'
+    // event sequences differ, and without the explicit re-convergence point the warp's threads
+    // drift apart and issue their events one subset at a time.
+    bool live = done < n_req;
+    while (__any_sync(wmask, live)) {
+        if (live) {
+            do {
+                if (!idle && (i >= n_req || busy < next_a)) {
+                    now = busy;                                   // block end
+                    if (run_last) {
+                        __stcs(te + run_req * st, now - run_arr);
+                        ++done;
+                    }
+                    idle = true;
+                    dispatch();
+                } else {
+                    now = next_a;                                 // arrival (first on ties)
+                    if (now < prev_a || now < 0 || next_t >= a.n_types) { err = 1u; break; }
+                    prev_a = now;
+                    const uint32_t m = next_t, e = s_ext[m];
+                    uint32_t pos = n, left0 = e, tb0 = m;
+                    if (a.policy != 0u) {
+                        // Algorithm 1 (R12): scan from the tail; stay behind the first request of
+                        // the same type or with Ext_left * Ext <= Ext_left(new) * Ext(new)
+                        const uint64_t key = (uint64_t)e * e;
+                        pos = 0;
+                        for (uint32_t j = n; j-- > 0;) {
+                            const uint32_t tj = Q(q_tb, j) & 0xFFFFu;
+                            if (tj == m || (uint64_t)Q(q_left, j) * s_ext[tj] <= key) { pos = j + 1; break; }
+                        }
+                    }
+                    if (a.policy == 2u) {
+                        // f4 elastic splitting (R23): suspended under high density or many requests of the
+                        // same type -> unsplit, at the tail
+                        uint32_t same = 0;
+                        for (uint32_t j = 0; j < n; ++j) same += ((Q(q_tb, j) & 0xFFFFu) == m) ? 1u : 0u;
+                        const bool off = (n >= a.d_max) | (same >= a.s_max);
+                        pos = off ? n : pos;
+                        left0 = off ? s_uns[m] : e;
+                        tb0 = off ? (m | (kQosUnsplit << 16)) : m;
+                    }
+                    if (n == kQosQueue) { err = 2u; break; }
+                    for (uint32_t j = n; j > pos; --j) {
+                        Q(q_req, j) = Q(q_req, j - 1);
+                        Q(q_left, j) = Q(q_left, j - 1);
+                        Q(q_tb, j) = Q(q_tb, j - 1);
+                    }
+                    Q(q_req, pos) = i;
+                    Q(q_left, pos) = left0;
+                    Q(q_tb, pos) = tb0;
+                    ++n;
+                    ++i;
+                    if (i < n_req) {
+                        next_a = __ldcs(arr + i * st);
+                        next_t = __ldcs(ty + i * st);
+                    }
+                    dispatch();
                 }
-            }
-            if (n == kQosQueue) { err = 2u; break; }
-            for (uint32_t j = n; j > pos; --j) {
-                Q(q_req, j) = Q(q_req, j - 1);
-                Q(q_left, j) = Q(q_left, j - 1);
-                Q(q_tb, j) = Q(q_tb, j - 1);
-            }
-            Q(q_req, pos) = i;
-            Q(q_left, pos) = e;
-            Q(q_tb, pos) = m;
-            ++n;
-            ++i;
-            if (i < n_req) {
-                next_a = __ldcs(arr + i * st);
-                next_t = __ldcs(ty + i * st);
-            }
-            dispatch();
+            } while (0);
+            live = (err == 0u) && (done < n_req);
         }
+        __syncwarp(wmask);
     }
 #undef Q
     if (err) {
@@ -145,7 +172,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
 size_t qos_smem_bytes(const QosArgs& a)
 {
     return 4 * ((size_t)2 * a.n_types + 1 + a.n_alpha + a.n_blocks_total) + 4 * (size_t)3 * kQosQueue * kQosThreads +
-           4 * (size_t)a.n_alpha * kQosThreads + 16;
+           4 * (size_t)a.n_alpha * kQosThreads + 4 * (size_t)a.n_types + 16;
 }
 
 cudaError_t launch_qos(const QosArgs& a, cudaStream_t st)

@@ -87,6 +87,10 @@ def _load():
         "split_qos_simulate": (C.c_int, [P(C.c_int64), P(C.c_uint32), C.c_uint32, C.c_uint32, P(C.c_uint32),
                                          C.c_uint32, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p, C.c_void_p,
                                          C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),
+        "split_qos_simulate_elastic": (C.c_int, [P(C.c_int64), P(C.c_uint32), P(C.c_int64), C.c_uint32, C.c_uint32,
+                                                 C.c_uint32, P(C.c_uint32), C.c_uint32, C.c_uint64, C.c_uint32,
+                                                 C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int,
+                                                 C.c_void_p]),
         "split_comm_unique_id": (C.c_int, [C.c_void_p]),
         "split_comm_init": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, P(C.c_void_p)]),
         "split_comm_destroy": (None, [C.c_void_p]),
@@ -111,7 +115,8 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_eval_batch_host", "split_ga_run", "split_ga_population", "split_preempt_decide",
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
-            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain", "split_k_sweep")
+            "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain", "split_k_sweep",
+            "split_qos_simulate_elastic")
 
 
 def lib():
@@ -150,12 +155,15 @@ def split_preempt_decide(now_ns: int, alpha: float, queue, incoming) -> int:
     return int(pos.value)
 
 
-def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int = 0, stream=None):
+def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int = 0, stream=None,
+                       unsplit=None, d_max: int = 0, s_max: int = 0):
     """f2 QoS simulator (include/split_ga.h).  blocks: per model type, its block
     times (ns); arrival: device int64 tensor [n_req, n_rep] (request-major);
     type_id: device int32 tensor of the same shape.  Returns device tensors
     (t_ete [n_req, n_rep] int64, violations [n_rep, n_alpha] int32 (uint32 bits),
-    rr [n_rep, 2] f64)."""
+    rr [n_rep, 2] f64).  policy 2 = f4 elastic splitting
+    (split_qos_simulate_elastic): unsplit = per-type unsplit latency (ns),
+    d_max / s_max = the density and same-type thresholds (R23)."""
     import torch
     n_req, n_rep = arrival.shape
     flat = np.ascontiguousarray(np.concatenate([np.asarray(b, dtype=np.int64) for b in blocks]))
@@ -167,6 +175,17 @@ def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *
     rr = torch.empty((n_rep, 2), dtype=torch.float64, device=dev)
     assert arrival.dtype == torch.int64 and arrival.is_contiguous()
     assert type_id.dtype == torch.int32 and type_id.is_contiguous() and type_id.shape == arrival.shape
+    if policy == 2:
+        un = np.ascontiguousarray(np.asarray(unsplit, dtype=np.int64))
+        assert un.shape == (len(blocks),)
+        _check(lib().split_qos_simulate_elastic(flat.ctypes.data_as(C.POINTER(C.c_int64)),
+                                                nb.ctypes.data_as(C.POINTER(C.c_uint32)),
+                                                un.ctypes.data_as(C.POINTER(C.c_int64)), len(blocks), d_max, s_max,
+                                                al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep, n_req,
+                                                arrival.data_ptr(), type_id.data_ptr(), t_ete.data_ptr(),
+                                                viol.data_ptr(), rr.data_ptr(), device, _stream_handle(stream)),
+               "split_qos_simulate_elastic")
+        return t_ete, viol, rr
     _check(lib().split_qos_simulate(flat.ctypes.data_as(C.POINTER(C.c_int64)), nb.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     len(blocks), policy, al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep,
                                     n_req, arrival.data_ptr(), type_id.data_ptr(), t_ete.data_ptr(), viol.data_ptr(),

@@ -104,3 +104,76 @@ def test_error_paths(S):
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate([[0]], a, t, [2000], 0)                        # zero-length block
     assert e.value.code == S.SPLIT_E_RANGE
+
+
+# ---- f4 elastic splitting (split_qos_simulate_elastic, R23) ----
+
+BIG = (1 << 32) - 1
+
+
+def _run_el(S, blocks, uns, d, s, arr, ty, alphas=ALPHAS):
+    a = torch.from_numpy(np.ascontiguousarray(arr.T)).cuda()
+    t = torch.from_numpy(np.ascontiguousarray(ty.T)).cuda()
+    te, viol, rr = S.split_qos_simulate(blocks, a, t, alphas, 2, unsplit=uns, d_max=d, s_max=s)
+    torch.cuda.synchronize()
+    return np.ascontiguousarray(te.cpu().numpy().T), viol.cpu().numpy().view(np.uint32), rr.cpu().numpy()
+
+
+def _check_el(blocks, uns, d, s, arr, ty, te, viol, rr, alphas=ALPHAS):
+    a = [int(x) for x in arr]
+    t = [int(x) for x in ty]
+    want = Q.simulate(blocks, a, t, Q.ELASTIC, uns, d, s)
+    assert [int(x) for x in te] == want
+    v, rs, rq = Q.stats(blocks, t, want, alphas)
+    assert [int(x) for x in viol[:len(alphas)]] == v
+    assert rr[0] == rs and rr[1] == rq
+
+
+@pytest.mark.parametrize("d,s", [(0, BIG), (2, BIG), (BIG, 1), (3, 2), (BIG, BIG)])
+@pytest.mark.parametrize("seed", [3, 2023])
+def test_elastic_small_cases_all_replicas(S, d, s, seed):
+    blocks = wl.random_blocks(5, seed=seed, k_hi=6, lo=300_000, hi=9_000_000)
+    uns = [max(1, sum(b) - 150_000 * (len(b) - 1)) for b in blocks]     # no cut overheads
+    arr, ty = wl.qos_requests(37, 150, 30_000_000, 5, seed=seed)
+    te, viol, rr = _run_el(S, blocks, uns, d, s, arr, ty)
+    for r in range(arr.shape[0]):
+        _check_el(blocks, uns, d, s, arr[r], ty[r], te[r], viol[r], rr[r])
+    if d == BIG and s == BIG:                 # no suspension: exactly policy 1
+        te1, _, _ = _run(S, blocks, arr, ty, Q.ALG1)
+        assert (te1 == te).all()
+
+
+def test_elastic_worked_examples(S):
+    blocks, uns = [[5, 5, 5], [2]], [13, 2]
+    one = lambda a, t, d, s: _run_el(S, blocks, uns, d, s, np.array([a], dtype=np.int64),
+                                     np.array([t], dtype=np.int32), [2000])[0][0].tolist()
+    assert one([0, 1], [0, 1], 1, BIG) == [15, 16]      # tests/test_oracle_qos.py, by hand
+    assert one([0, 1], [0, 1], 2, BIG) == [17, 6]
+    assert one([0, 1], [0, 0], BIG, 1) == [15, 27]
+    assert one([0, 1, 2], [0, 0, 1], BIG, 1) == [17, 29, 5]
+
+
+def test_elastic_table2_sized_run_sampled(S):
+    tot = [10_800_000, 13_200_000, 28_350_000, 67_500_000, 20_400_000]
+    rng = np.random.default_rng(13)
+    blocks = []
+    for T in tot:
+        w = rng.uniform(0.8, 1.2, size=4)
+        blocks.append([int(x) for x in np.floor(T * w / w.sum()).astype(np.int64)])
+    uns = [sum(b) - 3 * 400_000 for b in blocks]
+    arr, ty = wl.qos_requests(8192, 1000, 110_000_000, 5, seed=8)
+    te, viol, rr = _run_el(S, blocks, uns, 2, 3, arr, ty)
+    assert (te >= np.array(uns, dtype=np.int64)[ty]).all()
+    for r in (0, 4095, 8191):
+        _check_el(blocks, uns, 2, 3, arr[r], ty[r], te[r], viol[r], rr[r])
+
+
+def test_elastic_error_paths(S):
+    a = torch.zeros((2, 1), dtype=torch.int64, device="cuda")
+    t = torch.zeros((2, 1), dtype=torch.int32, device="cuda")
+    with pytest.raises(S.SplitError) as e:
+        S.split_qos_simulate([[5]], a, t, [2000], 2, unsplit=[0], d_max=1, s_max=1)   # unsplit time 0
+    assert e.value.code == S.SPLIT_E_RANGE
+    with pytest.raises(S.SplitError) as e:
+        S.split_qos_simulate([[5]], a, t, [2000], 3)                                   # no such policy
+    assert e.value.code == S.SPLIT_E_INVAL

@@ -9,4 +9,5 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:ga_kernel -s 1 -c 1 -o gpurun_out/prof_ga python tools/prof_driver.py ga 2 500 > gpurun_out/ncu_ga.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval_batch -s 1 -c 1 -o gpurun_out/prof_eval python tools/prof_driver.py eval 2 > gpurun_out/ncu_eval.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:qos_kernel -s 1 -c 1 -o gpurun_out/prof_qos python tools/prof_driver.py qos 2 > gpurun_out/ncu_qos.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:qos_kernel -s 1 -c 1 -o gpurun_out/prof_qos_el python tools/prof_driver.py qos_el 2 > gpurun_out/ncu_qos_el.log 2>&1
 ls -la gpurun_out | tail -14

@@ -23,15 +23,18 @@ def main(what: str, reps: int = 3, gens: int = 500):
         for _ in range(reps):
             h.eval_batch(bits, n_cand, out)
         torch.cuda.synchronize()
-    elif what == "qos":
+    elif what in ("qos", "qos_el"):
         blocks = [[3_575_000, 3_031_000, 3_231_000, 3_191_000], [4_005_000, 4_052_000, 3_984_000, 4_040_000],
                   [8_984_000, 8_747_000, 8_865_000, 8_990_000], [22_314_000, 21_125_000, 18_922_000, 19_467_000],
                   [6_124_000, 6_154_000, 6_078_000, 6_139_000]]
         arr, typ = wl.qos_requests(65536, 1000, 110_000_000, 5, seed=2023)
         da = torch.from_numpy(np.ascontiguousarray(arr.T)).cuda()
         dt = torch.from_numpy(np.ascontiguousarray(typ.T)).cuda()
+        kw = {}
+        if what == "qos_el":     # f4 elastic (R23), the bench's thresholds
+            kw = dict(unsplit=[sum(b) - 300_000 for b in blocks], d_max=3, s_max=2)
         for _ in range(reps):
-            S.split_qos_simulate(blocks, da, dt, [1000 * a for a in range(2, 21)], 1)
+            S.split_qos_simulate(blocks, da, dt, [1000 * a for a in range(2, 21)], 2 if kw else 1, **kw)
         torch.cuda.synchronize()
         return
     elif what == "ga_big":
