@@ -86,7 +86,9 @@ def main(tag):
     traffic = {}
     for name, rep, per in (("ga_kernel", "prof_ga.ncu-rep", "launch (one RUN segment = 500 generations of C2)"),
                            ("eval_batch_kernel", "prof_eval.ncu-rep", "launch (C5, 2^24 candidates)"),
-                           ("qos_kernel", "prof_qos.ncu-rep", "launch (f2: 65,536 replicas x 1000 requests)")):
+                           ("qos_kernel", "prof_qos.ncu-rep", "launch (f2: 65,536 replicas x 1000 requests)"),
+                           ("qos_kernel, f4 elastic", "prof_qos_el.ncu-rep",
+                            "launch (f4: the same workload, d_max = 3, s_max = 2)")):
         path = os.path.join(OUT, rep)
         if not os.path.exists(path):
             continue
