@@ -19,6 +19,9 @@
 
 namespace splitga {
 
+// kConverge: advance every replica of a warp by one event per loop trip and re-converge the warp
+// after it (policy 2; see the loop).  Policies 0/1 run the free-running loop, measured faster there.
+template <bool kConverge>
 __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
 {
     extern __shared__ __align__(16) uint8_t smem[];
@@ -83,11 +86,11 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
             Q(q_tb, 0) = tb + (1u << 16);
         }
     };
-    // One event per thread per warp-iteration, with the warp re-converged after each: the replicas'
-    // event sequences differ, and without the explicit re-convergence point the warp's threads
-    // drift apart and issue their events one subset at a time.
+    // kConverge: one event per thread per warp-iteration, with the warp re-converged after each: the
+    // replicas' event sequences differ, and under policy 2 the warp's threads otherwise drift apart and
+    // issue their events one subset at a time (4x the warp instructions, DESIGN.md f4).
     bool live = done < n_req;
-    while (__any_sync(wmask, live)) {
+    while (kConverge ? __any_sync(wmask, live) : live) {
         if (live) {
             do {
                 if (!idle && (i >= n_req || busy < next_a)) {
@@ -144,7 +147,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
             } while (0);
             live = (err == 0u) && (done < n_req);
         }
-        __syncwarp(wmask);
+        if (kConverge) __syncwarp(wmask);
     }
 #undef Q
     if (err) {
@@ -179,10 +182,11 @@ cudaError_t launch_qos(const QosArgs& a, cudaStream_t st)
 {
     if (a.n_rep == 0) return cudaSuccess;
     const size_t sm = qos_smem_bytes(a);
-    cudaError_t e = cudaFuncSetAttribute(qos_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    const auto kern = (a.policy == 2u) ? qos_kernel<true> : qos_kernel<false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
     const uint32_t grid = (uint32_t)((a.n_rep + kQosThreads - 1) / kQosThreads);
-    qos_kernel<<<grid, kQosThreads, sm, st>>>(a);
+    kern<<<grid, kQosThreads, sm, st>>>(a);
     return cudaGetLastError();
 }
 
