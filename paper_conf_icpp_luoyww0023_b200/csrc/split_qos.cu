@@ -70,11 +70,11 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
         const uint32_t b = (blk == kQosUnsplit) ? s_uns[m] : s_blk[s_off[m] + blk];
         const uint32_t left = Q(q_left, 0) - b;
         run_req = Q(q_req, 0);
-        run_arr = __ldg(arr + run_req * st);
         busy = now + b;
         idle = false;
         run_last = (left == 0u);
         if (run_last) {
+            run_arr = __ldg(arr + run_req * st);          // needed only when the request completes
             for (uint32_t j = 1; j < n; ++j) {
                 Q(q_req, j - 1) = Q(q_req, j);
                 Q(q_left, j - 1) = Q(q_left, j);
