@@ -120,3 +120,27 @@ def test_oracle_and_product_share_no_code():
                 "paper_conf_icpp_luoyww0023_b200/, include/split_ga.h", "").replace(
                 "(``paper_conf_icpp_luoyww0023_b200``)", ""), f
             assert "split_ga.h\"" not in txt and "split_internal" not in txt, f
+
+
+def test_qos_host_validation_without_gpu():
+    # host-side argument checks run before any CUDA call (n_rep = 0: nothing to launch)
+    import ctypes as C
+    L = S.lib()
+    blk = np.array([5, 5], dtype=np.int64)
+    nb = np.array([2], dtype=np.uint32)
+    al = np.array([2000], dtype=np.uint32)
+    P64, P32 = C.POINTER(C.c_int64), C.POINTER(C.c_uint32)
+
+    def el(uns, d=1, s=1):
+        u = None if uns is None else np.array(uns, dtype=np.int64).ctypes.data_as(P64)
+        return L.split_qos_simulate_elastic(blk.ctypes.data_as(P64), nb.ctypes.data_as(P32), u, 1, d, s,
+                                            al.ctypes.data_as(P32), 1, 0, 0, None, None, None, None, None, 0, None)
+
+    assert el([9]) == 0
+    assert el(None) == S.SPLIT_E_INVAL                  # elastic needs the unsplit latencies
+    assert el([0]) == S.SPLIT_E_RANGE                   # unsplit time out of [1, 2^32)
+    assert el([1 << 32]) == S.SPLIT_E_RANGE
+    base = lambda pol: L.split_qos_simulate(blk.ctypes.data_as(P64), nb.ctypes.data_as(P32), 1, pol,
+                                            al.ctypes.data_as(P32), 1, 0, 0, None, None, None, None, None, 0, None)
+    assert base(0) == 0 and base(1) == 0
+    assert base(2) == S.SPLIT_E_INVAL                   # policy 2 only through split_qos_simulate_elastic
