@@ -504,7 +504,7 @@ def main():
             quns.append(int(np.asarray(lq, dtype=np.int64).sum()))    # unsplit: T, no cut overheads
             with S.SplitGA(lq, oq, pop_size=4096, n_elite=64, k_min=4, k_max=4, device=local, stream=stream) as hq:
                 rq = hq.run(50, 1)
-            qb.append(S.block_times(lq, oq, rq["bits"]))
+            qb.append(S.split_block_times(lq, oq, rq["bits"]))
         arr, typ = wl.qos_requests(QOS_REPLICAS, 1000, 110_000_000, len(qb), seed=2023)
         da = torch.from_numpy(np.ascontiguousarray(arr.T)).to(dev)       # request-major
         dt = torch.from_numpy(np.ascontiguousarray(typ.T)).to(dev)

@@ -150,6 +150,25 @@ typedef struct {
 } split_queue_state;
 int split_preempt_decide(const split_queue_state* q, uint32_t* insert_pos);
 
+/* Block execution times of one split under the additive model of Eq. 2's
+ * fitness (R2, R3): block j runs operators c_{j-1}+1 .. c_j
+ * ("selects m-1 cut points to divide vanilla models into m blocks",
+ * P@20780-20831), its time is the sum of their profiled latencies
+ * (P@18308-18385) plus the overhead of the cut that starts it (the block after
+ * cut p pays cut_overhead_ns[p]; block 1 pays nothing).  Host only, no GPU:
+ * the f2 simulator's per-model block lists come from here.
+ *   latencies_ns     host, n_ops >= 2 entries, each >= 0
+ *   cut_overhead_ns  host, n_ops-1 entries >= 0, or NULL (all 0)
+ *   bits             host, ceil((n_ops-1)/64) words, the split's cut bitset
+ *                    (padding bits >= n_ops-1 ignored)
+ *   out_ns           host, `cap` entries: t_1 .. t_k
+ * *k receives the number of blocks (popcount + 1) even when it exceeds cap
+ * (then SPLIT_E_RANGE and out_ns holds the first cap blocks).
+ * SPLIT_E_INVAL: NULL pointer (out_ns may be NULL only when cap == 0),
+ * n_ops < 2 or a negative latency / overhead. */
+int split_block_times(const int64_t* latencies_ns, const int64_t* cut_overhead_ns, uint32_t n_ops,
+                      const uint64_t* bits, int64_t* out_ns, uint32_t cap, uint32_t* k);
+
 /* f2 — QoS simulator (R20).  Batched Monte-Carlo
  * of one edge executor serving requests of n_types split models: requests are
  * preempted only between blocks (§3.4, P@24400-26700), the queue order is
@@ -188,13 +207,18 @@ int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint3
  * preemption); otherwise it is split and placed by Algorithm 1 exactly as
  * split_qos_simulate policy 1.  Queued unsplit requests take part in later
  * Algorithm 1 scans with Ext_left = unsplit_ns[m].  Violations and response
- * ratios use the same per-type Ext (sum of the split blocks) as
- * split_qos_simulate, so the two are directly comparable; d_max = s_max =
- * UINT32_MAX reproduces policy 1, d_max = 0 a FIFO queue of unsplit models.
+ * ratios are taken against ref_ns[m]: NULL = the same per-type Ext (sum of the
+ * split blocks) as split_qos_simulate, so the two are directly comparable; or
+ * e.g. ref_ns = unsplit_ns for §5.2's isolated execution time of the model
+ * (then a request served unsplit has RR >= 1 and the target is alpha * T).
+ * d_max = s_max = UINT32_MAX reproduces policy 1, d_max = 0 a FIFO queue of
+ * unsplit models.
  *   unsplit_ns  host, n_types entries in [1, 2^32)
+ *   ref_ns      host, n_types entries in [1, 2^32), or NULL
  * Other arguments, layouts, synchronisation and errors: split_qos_simulate. */
 int split_qos_simulate_elastic(const int64_t* blocks_ns, const uint32_t* n_blocks, const int64_t* unsplit_ns,
-                               uint32_t n_types, uint32_t d_max, uint32_t s_max, const uint32_t* alpha_milli,
+                               const int64_t* ref_ns, uint32_t n_types, uint32_t d_max, uint32_t s_max,
+                               const uint32_t* alpha_milli,
                                uint32_t n_alpha, uint64_t n_rep, uint32_t n_req, const int64_t* arrival_ns,
                                const uint32_t* type_id, int64_t* t_ete_out, uint32_t* viol_out, double* rr_out,
                                int device, void* stream);
@@ -235,9 +259,13 @@ int split_ga_set_chain(split_ga_t* h, const int64_t* latencies_ns, const int64_t
  * Runs the fixed-k GA (k_min = k_max = k, `generations`, `seed`) for every k
  * in [k_lo, k_hi] (1 <= k_lo <= k_hi <= the handle's k_max) and reports each
  * run's best split: Eq. 2 fitness, Eq. 1's expected wait S2/(2 S1) of a short
- * request arriving during the model (P@17226-17827), overheads and V.
- * *k_best = the k whose best split has the smallest Eq. 1 wait (ties -> the
- * smaller k; 0 if no k has a feasible split).  out: host, k_hi-k_lo+1 entries.
+ * request arriving during the model (P@17226-17827), overheads, V, S1, S2 and
+ * the block-count criterion cost_ns = S2/(2 S1) + OV: the short request's wait
+ * plus the latency the cuts add to the split request itself ("an optimal
+ * number of splits exists and more blocks may not be beneficial",
+ * P@18542-18830).  *k_best = the k of minimum cost (compared exactly in
+ * integers; ties -> the smaller k; 0 if no k has a feasible split; cost_ns =
+ * +INF for an infeasible k).  out: host, k_hi-k_lo+1 entries.
  * Synchronous; the handle's own k range is restored afterwards. */
 typedef struct {
     uint32_t k;
@@ -245,6 +273,8 @@ typedef struct {
     double expected_wait_ns;
     uint64_t overhead_ns;
     int64_t var_num;
+    uint64_t s1, s2;
+    double cost_ns;
 } split_k_result;
 int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32_t generations, uint64_t seed,
                   split_k_result* out, uint32_t* k_best);
@@ -258,6 +288,21 @@ int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32_t generati
  * 1 <= k_max <= the handle's k_max (the create-time guard keeps every sum in
  * range).  Synchronous. */
 int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out);
+
+/* f1 — the two-cut map, synthetic analog of Fig. 2 (P@11560-12128: "the
+ * relationship of splitting overhead and standard deviation to position of cut
+ * points.  The X-axis and Y-axis show position of the first cut point and the
+ * second cut point"; §3.1 P@15908-16933).  For every pair of cut positions
+ * a <= b in [0, n_ops-2] the split with cuts {a, b} (3 blocks; a == b: the
+ * one-cut split {a}, 2 blocks) under the handle's chain: V = k S2 - S1^2
+ * (= k^2 sigma^2, exact), OV = the cut overheads (splitting overhead =
+ * OV / T, fn. 2) and the Eq. 2 fitness (no block-count restriction).
+ * Outputs: DEVICE buffers of (n_ops-1)^2 entries, row-major, entry [a][b] at
+ * a*(n_ops-1)+b, 8-byte aligned; a > b gets V = -1, OV = 0, fitness =
+ * -INFINITY; any output may be NULL.  Asynchronous on the handle's stream;
+ * caller-owned buffers.  SPLIT_E_INVAL when the handle's k_max < 3 (its
+ * create-time guards must cover two cuts). */
+int split_heatmap2(split_ga_t* h, int64_t* var_out, uint64_t* ov_out, double* fit_out);
 
 void split_ga_destroy(split_ga_t* h);
 const char* split_strerror(int code);

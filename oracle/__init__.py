@@ -79,6 +79,9 @@ def lib():
         L.or_count_fixed_k.restype = C.c_uint64
         L.or_ga_run.argtypes = [C.c_uint32, P64, P64, C.POINTER(GAParams), C.c_uint32, C.c_uint64,
                                 C.POINTER(GABest), PU64, PD]
+        L.or_heatmap2.argtypes = [C.c_uint32, P64, P64, P64, PU64, PD]
+        L.or_heatmap2.restype = None
+        L.or_ga_migrate.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, PU64, PD]
     return _lib
 
 
@@ -187,3 +190,26 @@ def ga_run(lat, ovh, generations: int, seed: int, *, pop_size, n_elite, tourname
         out["population"] = pop
         out["fitness_all"] = fit
     return out
+
+
+def heatmap2(lat, ovh):
+    """Two-cut map (Fig. 2 analog): (V, OV, fitness), each [n-1][n-1], entry [a][b] for a <= b."""
+    lat, ovh = _chain(lat, ovh)
+    m = len(lat) - 1
+    V = np.zeros((m, m), dtype=np.int64)
+    OV = np.zeros((m, m), dtype=np.uint64)
+    F = np.zeros((m, m), dtype=np.float64)
+    lib().or_heatmap2(len(lat), _p(lat, C.c_int64), _p(ovh, C.c_int64), _p(V, C.c_int64), _p(OV, C.c_uint64),
+                      _p(F, C.c_double))
+    return V, OV, F
+
+
+def ga_migrate(pop, fit, n_migrants: int, island_base: int = 0):
+    """One island-migration step (R16) on copies of pop [I][N][W] and fit [I][N]; returns (pop, fit)."""
+    pop = np.array(pop, dtype=np.uint64, copy=True, order="C")
+    fit = np.array(fit, dtype=np.float64, copy=True, order="C")
+    I, N, W = pop.shape
+    rc = lib().or_ga_migrate(W, N, I, n_migrants, island_base, _p(pop, C.c_uint64), _p(fit, C.c_double))
+    if rc != 0:
+        raise ValueError(f"or_ga_migrate rc={rc}")
+    return pop, fit

@@ -107,9 +107,12 @@ def simulate(blocks: list[list[int]], arrival: list[int], types: list[int], poli
     return t_ete
 
 
-def stats(blocks: list[list[int]], types: list[int], t_ete: list[int], alpha_milli: list[int]):
-    """(violations per alpha, rr_sum, rr_sq) in request order."""
-    ext = [sum(b) for b in blocks]
+def stats(blocks: list[list[int]], types: list[int], t_ete: list[int], alpha_milli: list[int],
+          ref: list[int] | None = None):
+    """(violations per alpha, rr_sum, rr_sq) in request order.  The latency
+    reference of type m is ref[m] when given (e.g. the isolated unsplit T of
+    §5.2, P@33300-33700), else Ext(m) = the sum of its split blocks (R20)."""
+    ext = [sum(b) for b in blocks] if ref is None else list(ref)
     viol = [0] * len(alpha_milli)
     rr_sum = 0.0
     rr_sq = 0.0

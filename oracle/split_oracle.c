@@ -186,6 +186,8 @@ void or_fitness_batch(uint32_t n, const int64_t* lat, const int64_t* ovh, const 
         f_out[c] = or_fitness_value(n, lat, ovh, bits + c * W, k_min, k_max);
 }
 
+static void set_bit(uint64_t* row, uint32_t p);
+
 /* ------------------------------------------------------------------------ */
 /* Orders.  R10: ranking (f desc, index asc); canonical best (f desc, bitset  */
 /* asc as a big-endian unsigned number, word W-1 most significant).           */
@@ -284,6 +286,39 @@ double or_fitness_from(uint32_t k, int64_t V, int64_t OV, int64_t T)
     double x = sqrt((double)V) / ((double)k * (double)T);
     double y = ((double)OV / (double)T) / (double)k;
     return -(or_dexp(x - 1.0) + or_dexp(y - 1.0));
+}
+
+/* The two-cut map, synthetic analog of Fig. 2 (P@11560-12128: "The X-axis and
+ * Y-axis show position of the first cut point and the second cut point"; (a)
+ * splitting overhead, (b) standard deviation of block execution time): for
+ * every pair of cut positions a <= b in [0, n-2], the split with cuts {a, b}
+ * (3 blocks; a == b is the one-cut split {a}, 2 blocks) scored by or_fitness
+ * with no block-count restriction.  Row-major [n-1][n-1] outputs at [a][b];
+ * entries a > b get V = -1, OV = 0, fitness = -INFINITY.  Any output may be NULL. */
+void or_heatmap2(uint32_t n, const int64_t* lat, const int64_t* ovh, int64_t* var_out, uint64_t* ov_out,
+                 double* fit_out)
+{
+    uint32_t m = n - 1, W = (n - 1 + 63) / 64;
+    uint64_t* bits = (uint64_t*)calloc(W, sizeof(uint64_t));
+    for (uint32_t a = 0; a < m; ++a)
+        for (uint32_t b = 0; b < m; ++b) {
+            size_t e = (size_t)a * m + b;
+            if (a > b) {
+                if (var_out) var_out[e] = -1;
+                if (ov_out) ov_out[e] = 0;
+                if (fit_out) fit_out[e] = -INFINITY;
+                continue;
+            }
+            memset(bits, 0, sizeof(uint64_t) * W);
+            set_bit(bits, a);
+            set_bit(bits, b);
+            or_stats st;
+            or_fitness(n, lat, ovh, bits, 1, n, &st);
+            if (var_out) var_out[e] = st.var_num;
+            if (ov_out) ov_out[e] = st.overhead;
+            if (fit_out) fit_out[e] = st.fitness;
+        }
+    free(bits);
 }
 
 /* Count the fixed-k candidates C(n-1, k-1) by visiting every one (A2). */
@@ -412,6 +447,54 @@ static int cmp_migrant(const void* a, const void* b)
     if (x->f < y->f) return 1;
     if (x->src != y->src) return x->src < y->src ? -1 : 1;
     return (x->rank < y->rank) ? -1 : (x->rank > y->rank);
+}
+
+/* Island migration (reading R16; the island model is the north star's, not
+ * the paper's).  Every island exports its top-K by the ranking order (f desc,
+ * index asc) -- rows and fitness, snapshotted before any island changes; each
+ * island sorts the FOREIGN migrants by (f desc, source island asc, rank asc)
+ * and writes the first K into its K worst slots, worst order = (f asc, index
+ * desc): the r-th worst slot receives the r-th best migrant.  pop: [I][N][W],
+ * fit: [I][N], island i's global id = island_base + i.  1 <= K <= N. */
+int or_ga_migrate(uint32_t W, uint32_t N, uint32_t I, uint32_t K, uint32_t island_base,
+                  uint64_t* pop, double* fit)
+{
+    if (I < 2 || K < 1 || K > N) return -1;
+    const size_t rowsz = sizeof(uint64_t) * W;
+    uint32_t* order = (uint32_t*)malloc(sizeof(uint32_t) * N);
+    migrant* all = (migrant*)malloc(sizeof(migrant) * (size_t)I * K);
+    uint64_t* snap = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)I * K * W);
+    for (uint32_t i = 0; i < I; ++i) {
+        for (uint32_t c = 0; c < N; ++c) order[c] = c;
+        g_sort_fit = fit + (size_t)i * N;
+        qsort(order, N, sizeof(uint32_t), cmp_rank);
+        for (uint32_t r = 0; r < K; ++r) {
+            migrant* mg = &all[(size_t)i * K + r];
+            memcpy(snap + ((size_t)i * K + r) * W, pop + ((size_t)i * N + order[r]) * W, rowsz);
+            mg->f = fit[(size_t)i * N + order[r]];
+            mg->src = island_base + i;
+            mg->rank = r;
+            mg->row = snap + ((size_t)i * K + r) * W;
+        }
+    }
+    migrant* foreign = (migrant*)malloc(sizeof(migrant) * (size_t)I * K);
+    for (uint32_t i = 0; i < I; ++i) {
+        uint32_t nf = 0;
+        for (uint32_t s = 0; s < I; ++s)
+            if (s != i) for (uint32_t r = 0; r < K; ++r) foreign[nf++] = all[(size_t)s * K + r];
+        qsort(foreign, nf, sizeof(migrant), cmp_migrant);
+        /* worst order: (f asc, index desc) = reverse of the ranking order */
+        for (uint32_t c = 0; c < N; ++c) order[c] = c;
+        g_sort_fit = fit + (size_t)i * N;
+        qsort(order, N, sizeof(uint32_t), cmp_rank);
+        for (uint32_t r = 0; r < K && r < nf; ++r) {
+            uint32_t slot = order[N - 1 - r];
+            memcpy(pop + ((size_t)i * N + slot) * W, foreign[r].row, rowsz);
+            fit[(size_t)i * N + slot] = foreign[r].f;
+        }
+    }
+    free(foreign); free(snap); free(all); free(order);
+    return 0;
 }
 
 typedef struct {
@@ -551,43 +634,11 @@ int or_ga_run(uint32_t n, const int64_t* lat, const int64_t* ovh, const or_ga_pa
         if (gf > f_improve) { f_improve = gf; last_improve = gen; }
         if (p->stall_generations > 0 && gen - last_improve >= p->stall_generations) break;
 
-        /* island migration (R16): top-K of every island, all-gathered; each island
-         * takes the K best foreign migrants into its K worst slots */
+        /* island migration (R16) */
         if (I > 1 && p->migration_interval > 0 && gen < generations) {
-            uint32_t K = p->n_migrants;
-            migrant* all = (migrant*)malloc(sizeof(migrant) * (size_t)I * K);
-            uint64_t* snap = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)I * K * W);
-            for (uint32_t i = 0; i < I; ++i) {
-                for (uint32_t c = 0; c < N; ++c) order[c] = c;
-                g_sort_fit = fit + (size_t)i * N;
-                qsort(order, N, sizeof(uint32_t), cmp_rank);
-                for (uint32_t r = 0; r < K; ++r) {
-                    migrant* mg = &all[(size_t)i * K + r];
-                    memcpy(snap + ((size_t)i * K + r) * W, pop + ((size_t)i * N + order[r]) * W, rowsz);
-                    mg->f = fit[(size_t)i * N + order[r]];
-                    mg->src = p->island_base + i;
-                    mg->rank = r;
-                    mg->row = snap + ((size_t)i * K + r) * W;
-                }
-            }
-            migrant* foreign = (migrant*)malloc(sizeof(migrant) * (size_t)I * K);
-            for (uint32_t i = 0; i < I; ++i) {
-                uint32_t nf = 0;
-                for (uint32_t s = 0; s < I; ++s)
-                    if (s != i) for (uint32_t r = 0; r < K; ++r) foreign[nf++] = all[(size_t)s * K + r];
-                qsort(foreign, nf, sizeof(migrant), cmp_migrant);
-                /* worst order: (f asc, index desc) = reverse of the ranking order */
-                for (uint32_t c = 0; c < N; ++c) order[c] = c;
-                g_sort_fit = fit + (size_t)i * N;
-                qsort(order, N, sizeof(uint32_t), cmp_rank);
-                for (uint32_t r = 0; r < K && r < nf; ++r) {
-                    uint32_t slot = order[N - 1 - r];
-                    memcpy(pop + ((size_t)i * N + slot) * W, foreign[r].row, rowsz);
-                    fit[(size_t)i * N + slot] = foreign[r].f;
-                }
+            or_ga_migrate(W, N, I, p->n_migrants, p->island_base, pop, fit);
+            for (uint32_t i = 0; i < I; ++i)
                 record_update(&g, &rec[i], pop + (size_t)i * N * W, fit + (size_t)i * N, N, gen);
-            }
-            free(foreign); free(snap); free(all);
         }
     }
 

@@ -52,6 +52,10 @@ int or_brute(uint32_t n, const int64_t* lat, const int64_t* ovh, uint32_t k_min,
              or_brute_result* res, int64_t* minV_per_k, uint64_t* argminV_per_k);
 int or_dp(uint32_t n, const int64_t* lat, int64_t delta, uint32_t k_max, int64_t* Vstar);
 uint64_t or_count_fixed_k(uint32_t n, uint32_t k);
+void or_heatmap2(uint32_t n, const int64_t* lat, const int64_t* ovh, int64_t* var_out, uint64_t* ov_out,
+                 double* fit_out);
+int or_ga_migrate(uint32_t W, uint32_t N, uint32_t I, uint32_t K, uint32_t island_base,
+                  uint64_t* pop, double* fit);
 int or_ga_run(uint32_t n, const int64_t* lat, const int64_t* ovh, const or_ga_params* p,
               uint32_t generations, uint64_t seed, or_ga_best* best,
               uint64_t* final_pop, double* final_fit);

@@ -354,8 +354,60 @@ __global__ void __launch_bounds__(1024) dp_kernel(const uint32_t* P /*[n+1]*/, c
 }
 
 // ------------------------------------------------------------------------
+// Two-cut map (f1, the synthetic analog of Fig. 2, P@11560-12128): entry
+// [a][b] (a <= b) of the row-major (n-1)^2 outputs is the split with cuts
+// {a, b} -- three blocks, or the one-cut split {a} on the diagonal -- with
+// its exact V = k S2 - S1^2, OV and Eq. 2 fitness; a > b: V = -1, OV = 0,
+// fitness = -inf.  One CTA row per a (blockIdx.y), threads over b: the
+// chain pairs {P[b+1], ovh[b]} are read coalesced, the three outputs are
+// written coalesced (the kernel is store-bound: 24 B per entry).
+// ------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) heatmap2_kernel(ChainDev ch, int64_t* __restrict__ var_out,
+                                                        uint64_t* __restrict__ ov_out, double* __restrict__ fit_out)
+{
+    const uint32_t m = ch.n - 1, a = blockIdx.y;
+    const uint2 pa = __ldg(ch.po + a);               // {P[a+1], ovh[a]}
+    for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b < m; b += gridDim.x * blockDim.x) {
+        const size_t e = (size_t)a * m + b;
+        int64_t V = -1;
+        uint64_t OV = 0;
+        double f = -CUDART_INF;
+        if (a <= b) {
+            const uint2 pb = __ldg(ch.po + b);
+            uint32_t k;
+            uint64_t S2;
+            if (a == b) {                            // one cut: blocks [0, a], [a+1, n-1] (+ ovh[a])
+                const uint32_t t1 = pa.x, t2 = ch.T - pa.x + pa.y;
+                S2 = (uint64_t)t1 * t1 + (uint64_t)t2 * t2;
+                OV = pa.y;
+                k = 2;
+            } else {                                 // R3: the block after cut p pays ovh[p]
+                const uint32_t t1 = pa.x, t2 = pb.x - pa.x + pa.y, t3 = ch.T - pb.x + pb.y;
+                S2 = (uint64_t)t1 * t1 + (uint64_t)t2 * t2 + (uint64_t)t3 * t3;
+                OV = (uint64_t)pa.y + pb.y;
+                k = 3;
+            }
+            const uint64_t S1 = (uint64_t)ch.T + OV;
+            V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+            f = eq2(k, V, OV, ch);
+        }
+        if (var_out) var_out[e] = V;
+        if (ov_out) ov_out[e] = OV;
+        if (fit_out) fit_out[e] = f;
+    }
+}
+
+// ------------------------------------------------------------------------
 // Launchers
 // ------------------------------------------------------------------------
+cudaError_t launch_heatmap2(const ChainDev& ch, int64_t* var_out, uint64_t* ov_out, double* fit_out, cudaStream_t st)
+{
+    const uint32_t m = ch.n - 1;
+    const uint32_t gx = (m + 255) / 256;
+    heatmap2_kernel<<<dim3(gx, m), 256, 0, st>>>(ch, var_out, ov_out, fit_out);
+    return cudaGetLastError();
+}
+
 size_t exh_smem_bytes(const ExhArgs& a)
 {
     const size_t rows = a.m - a.c + 1, nb = 1u << a.c, NW = kExhThreads / 32;

@@ -368,6 +368,16 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     if ((uint64_t)p.n_islands * p.pop_size >= (1ull << 32)) return fail(SPLIT_E_INVAL, "n_islands * pop_size must be < 2^32");
     if (p.n_islands > p.islands_per_device && !p.comm)
         return fail(SPLIT_E_INVAL, "islands span ranks but comm is NULL");
+    if (p.comm) {
+        // the all-gathers write world * islands_per_device slots at rank * islands_per_device:
+        // any other layout would make NCCL write past (or into the wrong slots of) the buffers
+        const SplitComm* c = (const SplitComm*)p.comm;
+        if (p.n_islands != (uint32_t)c->world * p.islands_per_device || p.island_id != (uint32_t)c->rank * p.islands_per_device)
+            return fail(SPLIT_E_INVAL, "comm of rank %d / world %d needs n_islands = world*islands_per_device and "
+                        "island_id = rank*islands_per_device (got %u, %u)", c->rank, c->world, p.n_islands, p.island_id);
+        if (c->device != p.device)
+            return fail(SPLIT_E_INVAL, "comm is bound to device %d, params.device is %d", c->device, p.device);
+    }
     const bool migrate = p.migration_interval > 0 && p.n_islands > 1;
     if (migrate && (p.n_migrants < 1 || p.n_migrants > p.pop_size - p.n_elite || p.n_migrants > kMaxElite))
         return fail(SPLIT_E_INVAL, "n_migrants must be in [1, min(N - E, %u)]", kMaxElite);
@@ -444,26 +454,28 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     {
         const uint32_t grid_max = (uint32_t)(ga_max_blocks_per_sm(h->W) * h->num_sms);
         if (grid_max < 2 * a.I) {
+            const int sms = h->num_sms;          // read before h is freed
             free_all(h);
             delete h;
-            return fail(SPLIT_E_INVAL, "too many islands per device for %d SMs", h->num_sms);
+            return fail(SPLIT_E_INVAL, "too many islands per device for %d SMs", sms);
         }
         a.cpi = (grid_max - a.I) / a.I;
         a.cpi_pad = (a.cpi + 3u) & ~3u;
         a.stage_bits = (size_t)a.cpi_pad * h->W * 8 <= 16384 ? 1u : 0u;
     }
-    if (ga_smem_bytes(a) > 227 * 1024) {
+    if (const size_t smem = ga_smem_bytes(a); smem > 227 * 1024) {
         free_all(h);
         delete h;
         return fail(SPLIT_E_INVAL, "shared-memory plan %zu B exceeds 227 KB (n_ops, islands or migrants too large)",
-                    ga_smem_bytes(a));
+                    smem);
     }
     cudaError_t ge;
     h->grid = ga_grid(a, h->num_sms, &ge);
     if (ge != cudaSuccess || h->grid < 2 * (int)a.I) {
+        const int grid = h->grid;               // read before h is freed
         free_all(h);
         delete h;
-        return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s (grid %d)", cudaGetErrorString(ge), h->grid);
+        return fail(SPLIT_E_CUDA, "GA kernel occupancy: %s (grid %d)", cudaGetErrorString(ge), grid);
     }
     a.cpi = (uint32_t)(h->grid - (int)a.I) / a.I;     // <= the sizing value; cpi_pad keeps its value
     h->cpi = a.cpi;
@@ -551,13 +563,29 @@ extern "C" int split_ga_set_chain(split_ga_t* h, const int64_t* lat, const int64
     return SPLIT_OK;
 }
 
-// f3: Eq. 1-driven choice of the block count.  Eq. 1 (P@17226-17827) gives the
-// expected wait of a short request arriving during the split model as
-// S2 / (2 S1) = (sigma^2/t_bar + t_bar) / 2; more blocks shrink t_bar but add
-// overhead to S1, so the wait has a minimum over k ("an optimal number of
-// splits exists", P@18542-18830).  One fixed-k GA run per k in [k_lo, k_hi]
-// (same seed, same generation budget), then k* = argmin of the Eq. 1 wait of
-// each run's best split (ties -> smaller k; k without a feasible split skipped).
+// f3: Eq. 1-driven choice of the block count (reading R21).  Eq. 1
+// (P@17226-17827) gives the expected wait of a short request arriving while the
+// split model runs, S2 / (2 S1) = (sigma^2/t_bar + t_bar) / 2: more blocks shrink
+// t_bar, but every cut adds its overhead to the split request itself ("the
+// relationship between splitting overhead and average latency is hyperbolic,
+// indicating that an optimal number of splits exists and more blocks may not be
+// beneficial", P@18542-18830).  The criterion of a k is therefore
+//     J(k) = S2/(2 S1) + OV        (short request's Eq. 1 wait + the long one's added latency)
+// of the best split the fixed-k GA finds for it (same seed and budget per k);
+// k* = argmin J, ties -> the smaller k, k without a feasible split skipped.  The
+// comparison is exact: J = (S2 + 2 S1 OV) / (2 S1), cross-multiplied in 128 bits
+// (S2 < 2^63, S1 OV < 2^64, S1 < 2^32).  With a constant per-cut overhead
+// delta, S1 = T + (k-1) delta and OV = (k-1) delta are fixed per k, so J is
+// minimised by the minimum-S2 split and k* equals the exact DP's whenever every
+// run reaches the DP optimum.
+static bool kcost_less(uint64_t s2a, uint64_t s1a, uint64_t ova, uint64_t s2b, uint64_t s1b, uint64_t ovb)
+{
+    const unsigned __int128 na = (unsigned __int128)s2a + 2 * (unsigned __int128)s1a * ova;
+    const unsigned __int128 nb = (unsigned __int128)s2b + 2 * (unsigned __int128)s1b * ovb;
+    // na / (2 s1a) < nb / (2 s1b)  <=>  na * s1b < nb * s1a  (all < 2^97)
+    return na * s1b < nb * s1a;
+}
+
 extern "C" int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32_t generations, uint64_t seed,
                              split_k_result* out, uint32_t* k_best)
 {
@@ -568,7 +596,7 @@ extern "C" int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32
     std::vector<uint64_t> bits(h->W ? h->W : 1);
     int rc = SPLIT_OK;
     *k_best = 0;
-    double best_wait = 0.0;
+    uint64_t b_s2 = 0, b_s1 = 1, b_ov = 0;
     for (uint32_t k = k_lo; k <= k_hi && rc == SPLIT_OK; ++k) {
         h->ch.k_min = h->ch.k_max = k;
         h->ga.ch.k_min = h->ga.ch.k_max = k;
@@ -583,9 +611,15 @@ extern "C" int split_k_sweep(split_ga_t* h, uint32_t k_lo, uint32_t k_hi, uint32
         r.expected_wait_ns = b.expected_wait_ns;
         r.overhead_ns = b.overhead_ns;
         r.var_num = b.var_num;
-        if (b.fitness > -INFINITY && (*k_best == 0 || b.expected_wait_ns < best_wait)) {
+        r.s1 = b.s1;
+        r.s2 = b.s2;
+        const bool feasible = b.fitness > -INFINITY;
+        r.cost_ns = feasible ? b.expected_wait_ns + (double)b.overhead_ns : INFINITY;
+        if (feasible && (*k_best == 0 || kcost_less(b.s2, b.s1, b.overhead_ns, b_s2, b_s1, b_ov))) {
             *k_best = k;
-            best_wait = b.expected_wait_ns;
+            b_s2 = b.s2;
+            b_s1 = b.s1;
+            b_ov = b.overhead_ns;
         }
     }
     h->ch.k_min = h->ga.ch.k_min = kmin0;
@@ -612,6 +646,7 @@ extern "C" int split_eval_batch(split_ga_t* h, const uint64_t* bits, uint64_t n_
     if (!bits || !out) return fail(SPLIT_E_INVAL, "split_eval_batch: NULL buffer");
     if (((uintptr_t)bits & 15u) || ((uintptr_t)out & 7u)) return fail(SPLIT_E_ALIGN, "bitsets must be 16-byte aligned, fitness 8-byte");
     cudaPointerAttributes at;
+    memset(&at, 0, sizeof(at));             // a failed query leaves it untouched: type reads as unregistered
     if (cudaPointerGetAttributes(&at, bits) != cudaSuccess || at.type != cudaMemoryTypeDevice) {
         cudaGetLastError();
         if (!(at.type == cudaMemoryTypeManaged)) return fail(SPLIT_E_INVAL, "cut_bitsets is not a device pointer");
@@ -916,6 +951,35 @@ extern "C" int split_preempt_decide(const split_queue_state* q, uint32_t* insert
 }
 
 // ------------------------------------------------------------------------
+// block times of a split (host; R2, R3): the block after cut p pays ovh[p]
+// ------------------------------------------------------------------------
+extern "C" int split_block_times(const int64_t* lat, const int64_t* ovh, uint32_t n, const uint64_t* bits,
+                                 int64_t* out_ns, uint32_t cap, uint32_t* k)
+{
+    if (!lat || !bits || !k || (cap > 0 && !out_ns)) return fail(SPLIT_E_INVAL, "split_block_times: NULL argument");
+    if (n < 2) return fail(SPLIT_E_INVAL, "split_block_times: n_ops must be >= 2");
+    for (uint32_t i = 0; i < n; ++i)
+        if (lat[i] < 0) return fail(SPLIT_E_INVAL, "latencies_ns[%u] < 0", i);
+    if (ovh)
+        for (uint32_t i = 0; i + 1 < n; ++i)
+            if (ovh[i] < 0) return fail(SPLIT_E_INVAL, "cut_overhead_ns[%u] < 0", i);
+    uint32_t j = 0;
+    int64_t cur = 0;
+    for (uint32_t p = 0; p < n; ++p) {
+        cur += lat[p];
+        const bool cut = p + 1 < n && ((bits[p >> 6] >> (p & 63)) & 1ull);
+        if (cut || p + 1 == n) {
+            if (j < cap) out_ns[j] = cur;
+            ++j;
+            cur = cut ? (ovh ? ovh[p] : 0) : 0;
+        }
+    }
+    *k = j;
+    if (j > cap) return fail(SPLIT_E_RANGE, "split_block_times: %u blocks > cap %u", j, cap);
+    return SPLIT_OK;
+}
+
+// ------------------------------------------------------------------------
 // device self-tests
 // ------------------------------------------------------------------------
 extern "C" int split_selftest_philox(int device, const uint32_t* in, uint32_t n, uint32_t* out)
@@ -1092,6 +1156,20 @@ extern "C" int split_exhaustive(split_ga_t* h, split_best_t* best_out, int64_t* 
     return SPLIT_OK;
 }
 
+extern "C" int split_heatmap2(split_ga_t* h, int64_t* var_out, uint64_t* ov_out, double* fit_out)
+{
+    if (!h) return fail(SPLIT_E_INVAL, "split_heatmap2: NULL handle");
+    if (h->p.k_max < 3 && h->n > 2)
+        return fail(SPLIT_E_INVAL, "split_heatmap2: the handle's k_max must be >= 3 (its guards cover two cuts)");
+    if (((uintptr_t)var_out | (uintptr_t)ov_out | (uintptr_t)fit_out) & 7u)
+        return fail(SPLIT_E_ALIGN, "split_heatmap2: outputs must be 8-byte aligned");
+    if (!var_out && !ov_out && !fit_out) return SPLIT_OK;
+    CU(cudaSetDevice(h->device));
+    CU(launch_heatmap2(h->ch, var_out, ov_out, fit_out, h->stream));
+    h->stats.launches = 1;
+    return SPLIT_OK;
+}
+
 extern "C" int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out)
 {
     if (!h || !s2_out) return fail(SPLIT_E_INVAL, "split_dp_min_s2: NULL argument");
@@ -1116,7 +1194,8 @@ extern "C" int split_dp_min_s2(split_ga_t* h, uint32_t k_max, uint64_t* s2_out)
 // f2: QoS simulator (split_qos.cu)
 // ------------------------------------------------------------------------
 static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
-                        const int64_t* unsplit_ns, uint32_t d_max, uint32_t s_max, const uint32_t* alpha_milli,
+                        const int64_t* unsplit_ns, const int64_t* ref_ns, uint32_t d_max, uint32_t s_max,
+                        const uint32_t* alpha_milli,
                         uint32_t n_alpha, uint64_t n_rep, uint32_t n_req, const int64_t* arrival_ns,
                         const uint32_t* type_id, int64_t* t_ete_out, uint32_t* viol_out, double* rr_out, int device,
                         void* stream)
@@ -1131,6 +1210,13 @@ static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint
             if (unsplit_ns[m] < 1 || unsplit_ns[m] >= ((int64_t)1 << 32))
                 return fail(SPLIT_E_RANGE, "split_qos_simulate_elastic: unsplit time out of [1, 2^32)");
             uns.push_back((uint32_t)unsplit_ns[m]);
+        }
+    std::vector<uint32_t> refv;
+    if (ref_ns)
+        for (uint32_t m = 0; m < n_types; ++m) {
+            if (ref_ns[m] < 1 || ref_ns[m] >= ((int64_t)1 << 32))
+                return fail(SPLIT_E_RANGE, "split_qos_simulate_elastic: ref_ns out of [1, 2^32)");
+            refv.push_back((uint32_t)ref_ns[m]);
         }
     if (n_alpha > kQosMaxAlpha || (n_alpha && !alpha_milli))
         return fail(SPLIT_E_INVAL, "split_qos_simulate: at most %u alpha thresholds", kQosMaxAlpha);
@@ -1162,6 +1248,8 @@ static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint
     tab.insert(tab.end(), alpha_milli, alpha_milli + n_alpha);
     tab.insert(tab.end(), blk.begin(), blk.end());
     tab.insert(tab.end(), uns.begin(), uns.end());
+    if (refv.empty()) refv = ext;                       // statistics against the split model's Ext (R20)
+    tab.insert(tab.end(), refv.begin(), refv.end());
     tab.push_back(0);                                   // error flag
     QosArgs a;
     memset(&a, 0, sizeof(a));
@@ -1193,6 +1281,7 @@ static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint
     a.alpha_milli = a.ext + n_types;
     a.blk_ns = a.alpha_milli + n_alpha;
     a.uns = a.blk_ns + blk.size();
+    a.ref = a.uns + uns.size();
     a.err = d_tab + tab.size() - 1;
     CU(launch_qos(a, st));
     uint32_t err = 0;
@@ -1209,18 +1298,18 @@ extern "C" int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_bl
                                   uint32_t* viol_out, double* rr_out, int device, void* stream)
 {
     if (policy > 1) return fail(SPLIT_E_INVAL, "split_qos_simulate: policy must be 0 (FIFO) or 1 (Algorithm 1)");
-    return qos_simulate(blocks_ns, n_blocks, n_types, policy, nullptr, 0, 0, alpha_milli, n_alpha, n_rep, n_req,
+    return qos_simulate(blocks_ns, n_blocks, n_types, policy, nullptr, nullptr, 0, 0, alpha_milli, n_alpha, n_rep, n_req,
                         arrival_ns, type_id, t_ete_out, viol_out, rr_out, device, stream);
 }
 
 extern "C" int split_qos_simulate_elastic(const int64_t* blocks_ns, const uint32_t* n_blocks, const int64_t* unsplit_ns,
-                                          uint32_t n_types, uint32_t d_max, uint32_t s_max,
+                                          const int64_t* ref_ns, uint32_t n_types, uint32_t d_max, uint32_t s_max,
                                           const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep,
                                           uint32_t n_req, const int64_t* arrival_ns, const uint32_t* type_id,
                                           int64_t* t_ete_out, uint32_t* viol_out, double* rr_out, int device,
                                           void* stream)
 {
     if (!unsplit_ns) return fail(SPLIT_E_INVAL, "split_qos_simulate_elastic: NULL unsplit_ns");
-    return qos_simulate(blocks_ns, n_blocks, n_types, 2, unsplit_ns, d_max, s_max, alpha_milli, n_alpha, n_rep, n_req,
+    return qos_simulate(blocks_ns, n_blocks, n_types, 2, unsplit_ns, ref_ns, d_max, s_max, alpha_milli, n_alpha, n_rep, n_req,
                         arrival_ns, type_id, t_ete_out, viol_out, rr_out, device, stream);
 }

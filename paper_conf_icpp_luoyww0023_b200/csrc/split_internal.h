@@ -133,6 +133,7 @@ struct QosArgs {
     // requests of its own type, runs unsplit (one block of uns[type] ns) and joins the tail
     uint32_t d_max, s_max;
     const uint32_t* uns;           // [n_types] unsplit latency T per type (policy 2 only)
+    const uint32_t* ref;           // [n_types] latency reference of violations / RR (= ext unless the caller sets it)
 };
 size_t qos_smem_bytes(const QosArgs& a);
 cudaError_t launch_qos(const QosArgs& a, cudaStream_t st);
@@ -140,6 +141,7 @@ cudaError_t launch_qos(const QosArgs& a, cudaStream_t st);
 cudaError_t launch_exh_table(const ExhArgs& a, cudaStream_t st);
 cudaError_t launch_exh(const ExhArgs& a, int mode, uint32_t grid, cudaStream_t st);
 cudaError_t launch_exh_reduce(const void* res, uint32_t n, void* out, cudaStream_t st);
+cudaError_t launch_heatmap2(const ChainDev& ch, int64_t* var_out, uint64_t* ov_out, double* fit_out, cudaStream_t st);
 cudaError_t launch_dp(const uint32_t* P, const uint32_t* ovh, uint32_t n, uint32_t k_max, uint64_t* s2_out,
                       cudaStream_t st);
 

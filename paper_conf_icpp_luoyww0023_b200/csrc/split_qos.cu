@@ -35,12 +35,14 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     uint32_t* q_tb = q_left + kQosQueue * kQosThreads;    // type | next block << 16
     uint32_t* s_viol = q_tb + kQosQueue * kQosThreads;    // [n_alpha][kQosThreads]
     uint32_t* s_uns = s_viol + a.n_alpha * kQosThreads;   // [M] unsplit T (policy 2)
+    uint32_t* s_ref = s_uns + a.n_types;                  // [M] latency reference of the statistics
     for (uint32_t j = threadIdx.x; j <= a.n_types; j += blockDim.x) s_off[j] = a.blk_off[j];
     for (uint32_t j = threadIdx.x; j < a.n_types; j += blockDim.x) s_ext[j] = a.ext[j];
     for (uint32_t j = threadIdx.x; j < a.n_alpha; j += blockDim.x) s_alpha[j] = a.alpha_milli[j];
     for (uint32_t j = threadIdx.x; j < nb; j += blockDim.x) s_blk[j] = a.blk_ns[j];
     if (a.policy == 2u)
         for (uint32_t j = threadIdx.x; j < a.n_types; j += blockDim.x) s_uns[j] = a.uns[j];
+    for (uint32_t j = threadIdx.x; j < a.n_types; j += blockDim.x) s_ref[j] = a.ref[j];
     __syncthreads();
     const uint32_t tid = threadIdx.x;
     const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + tid;
@@ -159,7 +161,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     double rs = 0.0, rq = 0.0;
     for (uint32_t k = 0; k < n_req; ++k) {
         const int64_t t = __ldcs(te + k * st);
-        const uint32_t e = s_ext[__ldcs(ty + k * st)];
+        const uint32_t e = s_ref[__ldcs(ty + k * st)];     // Ext of the split model, or the caller's reference
         const uint64_t t1000 = 1000ull * (uint64_t)t;
         for (uint32_t j = 0; j < a.n_alpha; ++j)
             s_viol[j * kQosThreads + tid] += (t1000 > (uint64_t)s_alpha[j] * e) ? 1u : 0u;
@@ -175,7 +177,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
 size_t qos_smem_bytes(const QosArgs& a)
 {
     return 4 * ((size_t)2 * a.n_types + 1 + a.n_alpha + a.n_blocks_total) + 4 * (size_t)3 * kQosQueue * kQosThreads +
-           4 * (size_t)a.n_alpha * kQosThreads + 4 * (size_t)a.n_types + 16;
+           4 * (size_t)a.n_alpha * kQosThreads + 8 * (size_t)a.n_types + 16;
 }
 
 cudaError_t launch_qos(const QosArgs& a, cudaStream_t st)

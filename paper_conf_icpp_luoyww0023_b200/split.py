@@ -52,7 +52,8 @@ class split_queue_state(C.Structure):
 
 class split_k_result(C.Structure):
     _fields_ = [("k", C.c_uint32), ("fitness", C.c_double), ("expected_wait_ns", C.c_double),
-                ("overhead_ns", C.c_uint64), ("var_num", C.c_int64)]
+                ("overhead_ns", C.c_uint64), ("var_num", C.c_int64), ("s1", C.c_uint64), ("s2", C.c_uint64),
+                ("cost_ns", C.c_double)]
 
 
 class split_run_stats(C.Structure):
@@ -87,7 +88,7 @@ def _load():
         "split_qos_simulate": (C.c_int, [P(C.c_int64), P(C.c_uint32), C.c_uint32, C.c_uint32, P(C.c_uint32),
                                          C.c_uint32, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p, C.c_void_p,
                                          C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),
-        "split_qos_simulate_elastic": (C.c_int, [P(C.c_int64), P(C.c_uint32), P(C.c_int64), C.c_uint32, C.c_uint32,
+        "split_qos_simulate_elastic": (C.c_int, [P(C.c_int64), P(C.c_uint32), P(C.c_int64), P(C.c_int64), C.c_uint32, C.c_uint32,
                                                  C.c_uint32, P(C.c_uint32), C.c_uint32, C.c_uint64, C.c_uint32,
                                                  C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int,
                                                  C.c_void_p]),
@@ -102,6 +103,9 @@ def _load():
         "split_last_run_stats": (C.c_int, [C.c_void_p, P(split_run_stats)]),
         "split_exhaustive": (C.c_int, [C.c_void_p, P(split_best_t), C.c_void_p, C.c_void_p]),
         "split_dp_min_s2": (C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p]),
+        "split_heatmap2": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
+        "split_block_times": (C.c_int, [C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.c_uint32,
+                                        P(C.c_uint32)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -116,7 +120,7 @@ EXPORTED = ("split_ga_params_default", "split_ga_create", "split_words", "split_
             "split_comm_unique_id", "split_comm_init", "split_comm_destroy", "split_ga_destroy",
             "split_strerror", "split_last_error", "split_selftest_philox", "split_selftest_dexp",
             "split_last_run_stats", "split_exhaustive", "split_dp_min_s2", "split_qos_simulate", "split_ga_set_chain", "split_k_sweep",
-            "split_qos_simulate_elastic")
+            "split_qos_simulate_elastic", "split_block_times", "split_heatmap2")
 
 
 def lib():
@@ -155,17 +159,24 @@ def split_preempt_decide(now_ns: int, alpha: float, queue, incoming) -> int:
     return int(pos.value)
 
 
-def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int = 0, stream=None,
-                       unsplit=None, d_max: int = 0, s_max: int = 0):
+def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *, device: int | None = None,
+                       stream=None, unsplit=None, d_max: int = 0, s_max: int = 0, ref=None):
     """f2 QoS simulator (include/split_ga.h).  blocks: per model type, its block
     times (ns); arrival: device int64 tensor [n_req, n_rep] (request-major);
     type_id: device int32 tensor of the same shape.  Returns device tensors
     (t_ete [n_req, n_rep] int64, violations [n_rep, n_alpha] int32 (uint32 bits),
     rr [n_rep, 2] f64).  policy 2 = f4 elastic splitting
     (split_qos_simulate_elastic): unsplit = per-type unsplit latency (ns),
-    d_max / s_max = the density and same-type thresholds (R23)."""
+    d_max / s_max = the density and same-type thresholds (R23); ref = per-type
+    latency reference for violations and RR (None = the split Ext).
+    device defaults to arrival's device, stream to that device's current torch
+    stream (the one the output tensors are allocated on)."""
     import torch
     n_req, n_rep = arrival.shape
+    if device is None:
+        device = arrival.device.index if arrival.device.index is not None else torch.cuda.current_device()
+    if stream is None:
+        stream = torch.cuda.current_stream(device)
     flat = np.ascontiguousarray(np.concatenate([np.asarray(b, dtype=np.int64) for b in blocks]))
     nb = np.ascontiguousarray(np.array([len(b) for b in blocks], dtype=np.uint32))
     al = np.ascontiguousarray(np.asarray(alpha_milli, dtype=np.uint32))
@@ -178,13 +189,18 @@ def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *
     if policy == 2:
         un = np.ascontiguousarray(np.asarray(unsplit, dtype=np.int64))
         assert un.shape == (len(blocks),)
+        rf = None if ref is None else np.ascontiguousarray(np.asarray(ref, dtype=np.int64))
+        if rf is not None and rf.shape != (len(blocks),):
+            raise ValueError("ref needs one entry per model type")
         _check(lib().split_qos_simulate_elastic(flat.ctypes.data_as(C.POINTER(C.c_int64)),
                                                 nb.ctypes.data_as(C.POINTER(C.c_uint32)),
-                                                un.ctypes.data_as(C.POINTER(C.c_int64)), len(blocks), d_max, s_max,
+                                                un.ctypes.data_as(C.POINTER(C.c_int64)),
+                                                None if rf is None else rf.ctypes.data_as(C.POINTER(C.c_int64)),
+                                                len(blocks), d_max, s_max,
                                                 al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep, n_req,
                                                 arrival.data_ptr(), type_id.data_ptr(), t_ete.data_ptr(),
                                                 viol.data_ptr(), rr.data_ptr(), device, _stream_handle(stream)),
-               "split_qos_simulate_elastic")
+               "split_qos_simulate_elastic", "split_block_times", "split_heatmap2")
         return t_ete, viol, rr
     _check(lib().split_qos_simulate(flat.ctypes.data_as(C.POINTER(C.c_int64)), nb.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     len(blocks), policy, al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep,
@@ -193,19 +209,20 @@ def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *
     return t_ete, viol, rr
 
 
-def block_times(latencies_ns, cut_overhead_ns, bits) -> list[int]:
-    """Block execution times (ns) of a split under the additive model (R2, R3):
-    the block after cut p pays ovh[p].  bits: the split's W words (host)."""
-    lat = np.asarray(latencies_ns, dtype=np.int64)
-    ovh = np.zeros(len(lat) - 1, dtype=np.int64) if cut_overhead_ns is None else np.asarray(cut_overhead_ns, np.int64)
-    out, cur = [], 0
-    for p in range(len(lat)):
-        cur += int(lat[p])
-        if p < len(lat) - 1 and (int(bits[p >> 6]) >> (p & 63)) & 1:
-            out.append(cur)
-            cur = int(ovh[p])
-    out.append(cur)
-    return out
+def split_block_times(latencies_ns, cut_overhead_ns, bits) -> list[int]:
+    """Block execution times (ns) of one split (include/split_ga.h split_block_times)."""
+    lat = np.ascontiguousarray(latencies_ns, dtype=np.int64)
+    ovh = None if cut_overhead_ns is None else np.ascontiguousarray(cut_overhead_ns, dtype=np.int64)
+    b = np.ascontiguousarray(bits, dtype=np.uint64)
+    if ovh is not None and ovh.size != lat.size - 1:
+        raise ValueError("cut_overhead_ns needs n_ops - 1 entries")
+    if b.size < words(lat.size):
+        raise ValueError("bits needs ceil((n_ops-1)/64) words")
+    out = np.zeros(lat.size, dtype=np.int64)           # at most n_ops blocks
+    k = C.c_uint32(0)
+    _check(_lib.split_block_times(_ptr(lat), None if ovh is None else _ptr(ovh), lat.size, _ptr(b), _ptr(out),
+                                  out.size, C.byref(k)), "split_block_times")
+    return [int(x) for x in out[:k.value]]
 
 
 def split_comm_unique_id() -> bytes:
@@ -259,6 +276,8 @@ class SplitGA:
                 raise ValueError("cut_overhead_ns needs n_ops - 1 entries")
             p.cut_overhead_ns = self._ovh.ctypes.data_as(C.POINTER(C.c_int64))
         p.device = device
+        if stream is None:
+            stream = _current_stream(device)
         p.stream = C.c_void_p(_stream_handle(stream))
         p.comm = C.c_void_p(comm) if comm else None
         self.params = p
@@ -299,6 +318,10 @@ class SplitGA:
         """Replace the handle's chain (same n_ops): host arrays, uploaded on the handle's stream."""
         lat = np.ascontiguousarray(latencies_ns, dtype=np.int64)
         ovh = None if cut_overhead_ns is None else np.ascontiguousarray(cut_overhead_ns, dtype=np.int64)
+        if lat.size != self.n_ops:
+            raise ValueError(f"latencies_ns needs n_ops = {self.n_ops} entries (got {lat.size})")
+        if ovh is not None and ovh.size != self.n_ops - 1:
+            raise ValueError(f"cut_overhead_ns needs n_ops - 1 = {self.n_ops - 1} entries (got {ovh.size})")
         self._keep_chain = (lat, ovh)          # the copy is staged before the call returns; kept for clarity
         _check(_lib.split_ga_set_chain(self._h, lat.ctypes.data_as(C.POINTER(C.c_int64)),
                                        None if ovh is None else ovh.ctypes.data_as(C.POINTER(C.c_int64))),
@@ -329,6 +352,23 @@ class SplitGA:
             out["min_v_per_k"] = mv
             out["argmin_per_k"] = am
         return out
+
+    # f1: the two-cut map (Fig. 2 analog) into device tensors
+    def heatmap2(self, var_out=None, ov_out=None, fit_out=None):
+        """Returns (V int64, OV int64 (uint64 bits), fitness f64) device tensors of shape
+        [n_ops-1, n_ops-1], entry [a][b] for a <= b; pass tensors to reuse buffers."""
+        import torch
+        m = self.n_ops - 1
+        dev = torch.device("cuda", self.params.device)
+        var_out = torch.empty((m, m), dtype=torch.int64, device=dev) if var_out is None else var_out
+        ov_out = torch.empty((m, m), dtype=torch.int64, device=dev) if ov_out is None else ov_out
+        fit_out = torch.empty((m, m), dtype=torch.float64, device=dev) if fit_out is None else fit_out
+        for t in (var_out, ov_out, fit_out):
+            if t.numel() < m * m or not t.is_contiguous():
+                raise ValueError("heatmap2 outputs need (n_ops-1)^2 contiguous entries")
+        _check(_lib.split_heatmap2(self._h, C.c_void_p(_dev_ptr(var_out)), C.c_void_p(_dev_ptr(ov_out)),
+                                   C.c_void_p(_dev_ptr(fit_out))), "split_heatmap2")
+        return var_out, ov_out, fit_out
 
     # f1: min S2 per block count by the O(k n^2) DP
     def dp_min_s2(self, k_max: int) -> np.ndarray:
@@ -364,6 +404,18 @@ class SplitGA:
 
     def __exit__(self, *exc):
         self.close()
+
+
+def _current_stream(device: int):
+    """torch's current stream on `device` (where torch allocates the caller's
+    tensors); 0 (legacy default stream) when torch has no usable CUDA."""
+    try:
+        import torch
+        if torch.cuda.is_available():
+            return torch.cuda.current_stream(device)
+    except Exception:
+        pass
+    return 0
 
 
 def _stream_handle(stream) -> int:

@@ -131,15 +131,18 @@ def test_qos_host_validation_without_gpu():
     al = np.array([2000], dtype=np.uint32)
     P64, P32 = C.POINTER(C.c_int64), C.POINTER(C.c_uint32)
 
-    def el(uns, d=1, s=1):
+    def el(uns, d=1, s=1, ref=None):
         u = None if uns is None else np.array(uns, dtype=np.int64).ctypes.data_as(P64)
-        return L.split_qos_simulate_elastic(blk.ctypes.data_as(P64), nb.ctypes.data_as(P32), u, 1, d, s,
+        rf = None if ref is None else np.array(ref, dtype=np.int64).ctypes.data_as(P64)
+        return L.split_qos_simulate_elastic(blk.ctypes.data_as(P64), nb.ctypes.data_as(P32), u, rf, 1, d, s,
                                             al.ctypes.data_as(P32), 1, 0, 0, None, None, None, None, None, 0, None)
 
     assert el([9]) == 0
+    assert el([9], ref=[9]) == 0
     assert el(None) == S.SPLIT_E_INVAL                  # elastic needs the unsplit latencies
     assert el([0]) == S.SPLIT_E_RANGE                   # unsplit time out of [1, 2^32)
     assert el([1 << 32]) == S.SPLIT_E_RANGE
+    assert el([9], ref=[0]) == S.SPLIT_E_RANGE          # latency reference out of [1, 2^32)
     base = lambda pol: L.split_qos_simulate(blk.ctypes.data_as(P64), nb.ctypes.data_as(P32), 1, pol,
                                             al.ctypes.data_as(P32), 1, 0, 0, None, None, None, None, None, 0, None)
     assert base(0) == 0 and base(1) == 0

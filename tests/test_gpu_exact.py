@@ -117,3 +117,40 @@ def test_exhaustive_rejects_large_n(S):
     with _handle(S, lat, None, 2, 8) as h:
         with pytest.raises(S.SplitError):
             h.exhaustive()
+
+
+@pytest.mark.parametrize("name", ["c1", "vgg16", "resnet50_175", "synthetic_1024"])
+def test_heatmap2_matches_oracle(S, name):
+    """f1 two-cut map (Fig. 2 analog): every entry of the (n-1)^2 map -- V, OV and the Eq. 2
+    fitness bits -- equals the oracle's loop over or_fitness; synthetic_1024 (1023^2 entries,
+    4096 CTAs) is compared on a strided sample of rows."""
+    lat, ovh = wl.c1_chain() if name == "c1" else wl.chain(name)
+    m = len(lat) - 1
+    with S.SplitGA(lat, ovh, pop_size=4, n_elite=0, k_min=2, k_max=min(32, len(lat))) as h:
+        V, OV, F = h.heatmap2()
+        torch.cuda.synchronize()
+    V, OV, F = V.cpu().numpy(), OV.cpu().numpy().view(np.uint64), F.cpu().numpy()
+    if m <= 200:
+        rV, rOV, rF = oracle.heatmap2(lat, ovh)
+        assert np.array_equal(V, rV) and np.array_equal(OV, rOV)
+        assert np.array_equal(F.view(np.uint64), rF.view(np.uint64))
+    else:
+        for a in list(range(0, m, 97)) + [m - 2, m - 1]:
+            for b in range(m):
+                if a > b:
+                    assert V[a, b] == -1 and OV[a, b] == 0 and np.isneginf(F[a, b])
+                    continue
+                bits = np.zeros(oracle.words(len(lat)), np.uint64)
+                for c in {a, b}:
+                    bits[c >> 6] |= np.uint64(1 << (c & 63))
+                st = oracle.fitness(lat, ovh, bits)
+                assert V[a, b] == st["var_num"] and OV[a, b] == st["overhead"]
+                assert np.float64(F[a, b]).view(np.uint64) == np.float64(st["fitness"]).view(np.uint64)
+
+
+def test_heatmap2_guards(S):
+    lat, ovh = wl.c1_chain()
+    with S.SplitGA(lat, ovh, pop_size=4, n_elite=0, k_min=2, k_max=2) as h:
+        with pytest.raises(S.SplitError) as e:
+            h.heatmap2()
+        assert e.value.code == S.SPLIT_E_INVAL

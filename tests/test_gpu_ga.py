@@ -203,29 +203,43 @@ def test_set_chain_matches_fresh_handle(S):
     assert np.array_equal(_fbits(fit), _fbits(o["fitness_all"][0]))
 
 
-def test_k_sweep_eq1_choice(S):
+@pytest.mark.parametrize("name", ["c1", "vgg16"])
+def test_k_sweep_eq1_choice(S, name):
     """f3 (R21): split_k_sweep == one oracle fixed-k GA per k, and with a
-    constant per-cut overhead (S1 fixed per k) each k's best reaches the exact
-    minimum S2 of the DP, so the chosen k is the exact argmin of Eq. 1's wait
-    S2 / (2 S1) over k, computed here from the oracle DP."""
-    lat, ovh = wl.c1_chain(overhead="const")
+    constant per-cut overhead (S1 and OV fixed per k) each k's best reaches the
+    exact minimum S2 of the DP, so the chosen k is the exact argmin over k of
+    J(k) = S2/(2 S1) + OV (Eq. 1's wait plus the added latency, P@18542-18830)
+    computed here in rationals from the oracle DP -- an interior k (3) on both
+    chains, not the end of the range."""
+    from fractions import Fraction
+    if name == "c1":
+        lat, ovh = wl.c1_chain(overhead="const")
+        kw, G, k_hi = dict(pop_size=256, n_elite=4, k_min=2, k_max=12), 50, 12
+    else:
+        lat, _ = wl.chain("vgg16")
+        ovh, _ = wl.constant_overhead(lat)
+        kw, G, k_hi = dict(pop_size=4096, n_elite=64, k_min=2, k_max=16), 40, 16
     delta = int(ovh[0])
-    with S.SplitGA(lat, ovh, pop_size=256, n_elite=4, k_min=2, k_max=12) as h:
-        kb, res = h.k_sweep(2, 12, 50, 42)
+    with S.SplitGA(lat, ovh, **kw) as h:
+        kb, res = h.k_sweep(2, k_hi, G, 42)
         r_after = h.run(3, 1)                       # the handle's own k range is restored
-    o_after = oracle.ga_run(lat, ovh, 3, 1, pop_size=256, n_elite=4, k_min=2, k_max=12)
+    o_after = oracle.ga_run(lat, ovh, 3, 1, **kw)
     assert r_after["fitness"] == o_after["fitness"]
-    V = oracle.dp(lat, delta, 12)
+    V = oracle.dp(lat, delta, k_hi)
     T = int(lat.sum())
-    waits = {}
+    J = {}
     for r in res:
         k = r["k"]
-        o = oracle.ga_run(lat, ovh, 50, 42, pop_size=256, n_elite=4, k_min=k, k_max=k)
+        o = oracle.ga_run(lat, ovh, G, 42, **{**kw, "k_min": k, "k_max": k})
         assert r["fitness"] == o["fitness"] and r["var_num"] == o["var_num"]
+        assert r["s1"] == o["s1"] and r["s2"] == o["s2"] and r["overhead_ns"] == o["overhead"]
         assert r["expected_wait_ns"] == o["s2"] / (2.0 * o["s1"])
+        assert r["cost_ns"] == r["expected_wait_ns"] + float(o["overhead"])
         S1 = T + (k - 1) * delta
-        s2_min = (int(V[k]) + S1 * S1) // k
         assert (int(V[k]) + S1 * S1) % k == 0
-        waits[k] = s2_min / (2.0 * S1)
-        assert r["expected_wait_ns"] == waits[k]
-    assert kb == min(waits, key=lambda k: (waits[k], k))
+        s2_min = (int(V[k]) + S1 * S1) // k
+        assert r["s2"] == s2_min                    # the GA reached the DP optimum for this k
+        J[k] = Fraction(s2_min, 2 * S1) + (k - 1) * delta
+    k_star = min(J, key=lambda k: (J[k], k))
+    assert 2 < k_star < k_hi                        # the criterion has an interior optimum here
+    assert kb == k_star

@@ -111,20 +111,20 @@ def test_error_paths(S):
 BIG = (1 << 32) - 1
 
 
-def _run_el(S, blocks, uns, d, s, arr, ty, alphas=ALPHAS):
+def _run_el(S, blocks, uns, d, s, arr, ty, alphas=ALPHAS, ref=None):
     a = torch.from_numpy(np.ascontiguousarray(arr.T)).cuda()
     t = torch.from_numpy(np.ascontiguousarray(ty.T)).cuda()
-    te, viol, rr = S.split_qos_simulate(blocks, a, t, alphas, 2, unsplit=uns, d_max=d, s_max=s)
+    te, viol, rr = S.split_qos_simulate(blocks, a, t, alphas, 2, unsplit=uns, d_max=d, s_max=s, ref=ref)
     torch.cuda.synchronize()
     return np.ascontiguousarray(te.cpu().numpy().T), viol.cpu().numpy().view(np.uint32), rr.cpu().numpy()
 
 
-def _check_el(blocks, uns, d, s, arr, ty, te, viol, rr, alphas=ALPHAS):
+def _check_el(blocks, uns, d, s, arr, ty, te, viol, rr, alphas=ALPHAS, ref=None):
     a = [int(x) for x in arr]
     t = [int(x) for x in ty]
     want = Q.simulate(blocks, a, t, Q.ELASTIC, uns, d, s)
     assert [int(x) for x in te] == want
-    v, rs, rq = Q.stats(blocks, t, want, alphas)
+    v, rs, rq = Q.stats(blocks, t, want, alphas, ref)
     assert [int(x) for x in viol[:len(alphas)]] == v
     assert rr[0] == rs and rr[1] == rq
 
@@ -141,6 +141,21 @@ def test_elastic_small_cases_all_replicas(S, d, s, seed):
     if d == BIG and s == BIG:                 # no suspension: exactly policy 1
         te1, _, _ = _run(S, blocks, arr, ty, Q.ALG1)
         assert (te1 == te).all()
+
+
+@pytest.mark.parametrize("d,s", [(2, BIG), (3, 2)])
+def test_elastic_isolated_reference_all_replicas(S, d, s):
+    # violations and RR against the isolated unsplit T (§5.2, P@33300-33700) instead of the split Ext:
+    # the same schedule, a different denominator; a request served unsplit then has RR >= 1
+    blocks = wl.random_blocks(5, seed=7, k_hi=6, lo=300_000, hi=9_000_000)
+    uns = [max(1, sum(b) - 150_000 * (len(b) - 1)) for b in blocks]
+    arr, ty = wl.qos_requests(37, 150, 30_000_000, 5, seed=7)
+    te, viol, rr = _run_el(S, blocks, uns, d, s, arr, ty, ref=uns)
+    te0, _, _ = _run_el(S, blocks, uns, d, s, arr, ty)
+    assert (te == te0).all()
+    for r in range(arr.shape[0]):
+        _check_el(blocks, uns, d, s, arr[r], ty[r], te[r], viol[r], rr[r], ref=uns)
+    assert (rr[:, 0] >= 150 - 1e-9).all()       # every t_ete >= the isolated T of its type
 
 
 def test_elastic_worked_examples(S):

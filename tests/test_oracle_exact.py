@@ -70,3 +70,41 @@ def test_dp_constant_chain_even_split():
     for k in (1, 2, 3, 4, 5, 6, 10):
         assert v[k] == 0          # 60 divisible by k
     assert v[7] > 0
+
+
+@pytest.mark.parametrize("name", ["c1", "vgg16"])
+def test_heatmap2_pins(name):
+    """Two-cut map (Fig. 2 analog, P@11560-12128): each entry's sigma is numpy's population
+    std of the explicit block-time list (built here from cumulative sums, not from the oracle),
+    the overhead is the sum of the two cuts' overheads, the minimum over the upper triangle is
+    brute force's minimum V for 3 blocks and over the diagonal the one for 2 blocks."""
+    if name == "c1":
+        lat, ovh = wl.c1_chain()
+    else:
+        lat, ovh = wl.chain("vgg16")
+    n = len(lat)
+    m = n - 1
+    V, OV, F = oracle.heatmap2(lat, ovh)
+    cs = np.concatenate([[0], np.cumsum(lat)])
+    T = int(cs[-1])
+    rng = np.random.default_rng(1)
+    pairs = [(a, b) for a in range(m) for b in range(a, m)]
+    for a, b in (pairs if len(pairs) < 100 else [pairs[i] for i in rng.choice(len(pairs), 120, replace=False)]):
+        cuts = [a] if a == b else [a, b]
+        ends = [int(cs[c + 1]) for c in cuts] + [T]
+        starts = [0] + [int(cs[c + 1]) for c in cuts]
+        t = np.array([e - s for s, e in zip(starts, ends)], dtype=np.float64)
+        t[1:] += [float(ovh[c]) for c in cuts]
+        k = len(t)
+        assert math.isclose(math.sqrt(V[a, b]) / k, float(np.std(t)), rel_tol=1e-12, abs_tol=1e-6)
+        assert int(OV[a, b]) == sum(int(ovh[c]) for c in cuts)
+        x = math.sqrt(V[a, b]) / (k * T)
+        y = (int(OV[a, b]) / T) / k
+        assert math.isclose(F[a, b], -(math.exp(x - 1) + math.exp(y - 1)), rel_tol=1e-14)
+    lower = np.tril_indices(m, -1)
+    assert (V[lower] == -1).all() and (OV[lower] == 0).all() and np.isneginf(F[lower]).all()
+    if n <= 20:
+        b = oracle.brute(lat, ovh)
+        iu = np.triu_indices(m, 1)
+        assert V[iu].min() == b["minV_per_k"][3]
+        assert np.diag(V).min() == b["minV_per_k"][2]

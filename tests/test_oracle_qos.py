@@ -121,3 +121,12 @@ def test_elastic_infinite_thresholds_is_algorithm1():
         a = [int(x) for x in arr[r]]
         t = [int(x) for x in ty[r]]
         assert qos.simulate(blocks, a, t, qos.ELASTIC, uns, 1 << 30, 1 << 30) == qos.simulate(blocks, a, t, qos.ALG1)
+
+
+def test_stats_against_an_isolated_reference():
+    # §5.2 (P@33300-33700) measures response ratios against the isolated execution time; with
+    # ref = the unsplit T per type the same latencies give, by hand: RR = 17/13 and 6/2 = 3;
+    # at alpha = 2 only the second violates (6000 > 4000, 17000 <= 26000)
+    viol, rs, rq = qos.stats([[5, 5, 5], [2]], [0, 1], [17, 6], [1000, 2000, 3000], ref=[13, 2])
+    assert viol == [2, 1, 0]
+    assert rs == 17 / 13 + 3.0 and rq == (17 / 13) ** 2 + 9.0
