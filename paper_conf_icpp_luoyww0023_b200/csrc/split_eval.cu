@@ -1,7 +1,9 @@
 // split_eval.cu — K1 split_eval_batch (a2) and the small self-test kernels.
 // SPLIT (ICPP'23) Eq. 2 fitness over cut bitsets; see split_device.cuh for the
 // shared Philox / dexp / staging helpers and DESIGN.md §5 for the design.
+#include <cuda.h>
 #include <stdlib.h>
+#include <string.h>
 
 #include "split_device.cuh"
 
@@ -93,60 +95,115 @@ struct EvalCfg {
 // occupancy mask of one row (bit q <=> half q non-empty, padding masked)
 // EXACT: the sort key is the exact cut count (one POPC per half) instead of the
 // number of non-empty halves (always exact for W <= 4).
-template <int W, bool EXACT>
+// SWZ (W = 16 only): the chunk buffer was written by a tensor TMA with the
+// 128-byte swizzle -- 16-byte chunk c of row r sits at chunk c ^ (r & 7), and
+// here r & 7 == lane & 7 -- so step j reads physical chunk (j + lane) & 7
+// (conflict-free across each 8-lane phase) and files its nibble under the
+// logical chunk.
+// The half holding the last valid position (qfull, valid bits lastm) is
+// captured from the registers of the pass: its padding bits are masked in the
+// mask, and only a row whose padding bits are actually set writes the masked
+// half back (a rare, divergent store; an unconditional read-modify-write of
+// that half costs a 32-way bank conflict per warp: every lane's row has it in
+// the same bank).
+__device__ __forceinline__ uint32_t comp4(const uint4& v, uint32_t i)
+{
+    return i == 0 ? v.x : (i == 1 ? v.y : (i == 2 ? v.z : v.w));
+}
+
+template <int W, bool EXACT, bool SWZ>
 __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, uint32_t validocc, uint32_t qfull,
                                                   uint32_t lastm, uint32_t& cuts)
 {
     constexpr uint32_t H = 2 * W;
-    uint32_t occr = 0, pc = 0;
-    if constexpr (W % 2 == 0) {
-        constexpr uint32_t C = W / 2;            // 16-byte chunks per row
+    uint32_t occ = 0, pc = 0, vq = 0;
+    uint4 ctop = make_uint4(0u, 0u, 0u, 0u);     // SWZ: logical chunk 7 (halves 28..31)
+    if constexpr (SWZ) {
+        // logical chunk j sits at physical chunk j ^ (lane & 7): reading in logical order is already
+        // conflict-free across each 8-lane phase, and every nibble lands at a constant shift
+        static_assert(W == 16, "the swizzled layout is defined for 128-byte rows");
         const uint4* my4 = (const uint4*)my;
-        uint32_t cc = lane % C;
+        const uint32_t rsw = lane & 7u;
 #pragma unroll
-        for (uint32_t j = 0; j < C; ++j) {
-            const uint4 v = my4[cc];
-            cc = (cc + 1 == C) ? 0u : cc + 1;
-            occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1) | (min(v.z, 1u) << 2) | (min(v.w, 1u) << 3)) << (4 * j);
-            if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+        for (uint32_t j = 0; j < 8; ++j) {
+            const uint4 v = my4[j ^ rsw];
+            occ |= (min(v.x, 1u) | (min(v.y, 1u) << 1) | (min(v.z, 1u) << 2) | (min(v.w, 1u) << 3)) << (4 * j);
+            if constexpr (EXACT) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+            if (j == 7) ctop = v;                // for W = 16 the padding (qfull >= 30) lives in chunk 7
+        }
+        vq = comp4(ctop, qfull & 3u);
+        if constexpr (EXACT) {
+            // padding: halves above qfull (all in chunk 7 for W = 16: qfull >= 30) and the bits of qfull >= lastm
+#pragma unroll
+            for (uint32_t i = 0; i < 4; ++i) {
+                const uint32_t q = 28u + i;
+                const uint32_t hv = comp4(ctop, i);
+                pc -= (q > qfull) ? __popc(hv) : ((q == qfull && lastm) ? __popc(hv & ~lastm) : 0u);
+            }
         }
     } else {
-        const uint2* my2 = (const uint2*)my;
-        uint32_t cc = lane % W;
+        uint32_t occr = 0;
+        if constexpr (W % 2 == 0) {
+            constexpr uint32_t C = W / 2;            // 16-byte chunks per row
+            const uint4* my4 = (const uint4*)my;
+            uint32_t cc = lane % C;
 #pragma unroll
-        for (uint32_t j = 0; j < W; ++j) {
-            const uint2 v = my2[cc];
-            cc = (cc + 1 == W) ? 0u : cc + 1;
-            occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1)) << (2 * j);
-            if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y);
+            for (uint32_t j = 0; j < C; ++j) {
+                const uint4 v = my4[cc];
+                if (cc == (qfull >> 2)) vq = comp4(v, qfull & 3u);
+                cc = (cc + 1 == C) ? 0u : cc + 1;
+                occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1) | (min(v.z, 1u) << 2) | (min(v.w, 1u) << 3)) << (4 * j);
+                if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+            }
+        } else {
+            const uint2* my2 = (const uint2*)my;
+            uint32_t cc = lane % W;
+#pragma unroll
+            for (uint32_t j = 0; j < W; ++j) {
+                const uint2 v = my2[cc];
+                if (cc == (qfull >> 1)) vq = (qfull & 1u) ? v.y : v.x;
+                cc = (cc + 1 == W) ? 0u : cc + 1;
+                occr |= (min(v.x, 1u) | (min(v.y, 1u) << 1)) << (2 * j);
+                if constexpr (W <= 4 || EXACT) pc += __popc(v.x) + __popc(v.y);
+            }
         }
-    }
-    // bit 4j+i (2j+i) of occr is half 4((j+l)%C)+i: rotate into place
-    const uint32_t rot = (W % 2 == 0) ? 4u * (lane % (W / 2)) : 2u * (lane % W);
-    uint32_t occ;
-    if constexpr (H == 32) occ = __funnelshift_l(occr, occr, rot);
-    else occ = ((occr << rot) | (occr >> ((H - rot) % H))) & ((1u << H) - 1u);
-    if constexpr (W <= 4 || EXACT) {
-        // exact cut count (sort key); padding bits removed below
-        for (uint32_t q = qfull; q < H; ++q) pc -= __popc(my[q] & ~((q == qfull) ? lastm : 0u));
+        // bit 4j+i (2j+i) of occr is half 4((j+l)%C)+i: rotate into place
+        const uint32_t rot = (W % 2 == 0) ? 4u * (lane % (W / 2)) : 2u * (lane % W);
+        if constexpr (H == 32) occ = __funnelshift_l(occr, occr, rot);
+        else occ = ((occr << rot) | (occr >> ((H - rot) % H))) & ((1u << H) - 1u);
+        if constexpr (W <= 4 || EXACT) {
+            // exact cut count (sort key); padding bits removed (rare halves: read back)
+            for (uint32_t q = qfull + 1; q < H; ++q) pc -= __popc(my[q]);
+            if (lastm) pc -= __popc(vq & ~lastm);
+        }
     }
     occ &= validocc;                             // padding: positions >= n-1 live in halves >= qfull
     if (lastm) {
-        const uint32_t vq = my[qfull] & lastm;
-        my[qfull] = vq;
-        occ |= min(vq, 1u) << qfull;
+        const uint32_t vm = vq & lastm;
+        if (vm != vq) {                          // padding bits set: mask the stored half for the walk
+            const uint32_t off = SWZ ? ((qfull * 4u) ^ ((lane & 7u) << 4)) / 4u : qfull;
+            my[off] = vm;
+        }
+        occ |= min(vm, 1u) << qfull;
     }
     cuts = (W <= 4 || EXACT) ? pc : __popc(occ);
     return occ;
 }
 
-template <int W, int NW_, int RPT_, int NB_, int KEY_ = 0>
+// SWZ (W = 16): every chunk -- the ragged last one included (rows past n_cand
+// arrive zero-filled) -- is one or two tensor TMA copies (box: 32 halves x
+// CHUNK/nbox rows, 128-byte swizzle) described by `tmap`; the chunk buffer is
+// 1024-byte aligned as the swizzle requires.
+template <int W, int NW_, int RPT_, int NB_, int KEY_ = 0, bool SWZ = false>
 __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / NW_ : 1)) eval_batch_w_kernel(ChainDev ch, const uint64_t* __restrict__ bits,
-                                                                uint64_t n_cand, double* __restrict__ out)
+                                                                uint64_t n_cand, double* __restrict__ out,
+                                                                const __grid_constant__ CUtensorMap tmap)
 {
     using Cfg = EvalCfg<W, NW_, RPT_, NB_>;
     constexpr uint32_t RPT = Cfg::RPT;
     constexpr uint32_t H = Cfg::H, CHW = Cfg::CHW, NB = Cfg::NB, NT = Cfg::NT, kChunk = Cfg::CHUNK;
+    constexpr uint32_t kBoxes = (kChunk + 255u) / 256u, kBoxRows = kChunk / kBoxes;
+    static_assert(!SWZ || (W == 16 && kBoxRows * kBoxes == kChunk && NT % 8 == 0), "swizzled chunk geometry");
     extern __shared__ __align__(16) uint8_t smem[];
     // staged chain: po[p] = {P[p+1], ovh[p]} for cut positions p in [0, n-2]
     const uint2* spo = (const uint2*)smem;
@@ -155,6 +212,10 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
     uint32_t* s_hist = s_occ + kChunk;                   // [32] histogram of the sort keys
     uint16_t* s_perm = (uint16_t*)(s_hist + 32);         // [kChunk] sorted order | flags
     uint32_t* s_buf = (uint32_t*)(s_perm + kChunk);      // [NB][CHW] (16-byte aligned)
+    if constexpr (SWZ) {
+        const uint32_t a = smem_u32(s_buf);
+        s_buf = (uint32_t*)((uint8_t*)s_buf + (((a + 1023u) & ~1023u) - a));
+    }
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     if (tid == 0) {
         mbar_init(mbar + 1, 1);
@@ -166,14 +227,26 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
     const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
     const uint32_t validocc = (qfull >= 32u) ? ~0u : ((1u << qfull) - 1u);   // halves wholly inside [0, n-2]
     const uint32_t spo_s = opaque32(smem_u32(spo));
-    const uint64_t n_full = n_cand / kChunk;     // full chunks go through TMA
     const uint64_t n_chunks = (n_cand + kChunk - 1) / kChunk;
+    const uint64_t n_full = SWZ ? n_chunks : n_cand / kChunk;     // chunks that go through TMA
     uint64_t c = blockIdx.x;
     auto issue = [&](uint64_t cc, uint32_t b) {
         if (tid == 0 && cc < n_full) {
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             mbar_arrive_expect_tx(mbar + 1 + b, CHW * 4u);
-            bulk_g2s(s_buf + b * CHW, bits + cc * kChunk * W, CHW * 4u, mbar + 1 + b);
+            if constexpr (SWZ) {
+#pragma unroll
+                for (uint32_t x = 0; x < kBoxes; ++x) {
+                    const int32_t y = (int32_t)(cc * kChunk + x * kBoxRows);
+                    asm volatile(
+                        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                        ::"r"(smem_u32(s_buf + b * CHW + x * kBoxRows * H)), "l"(&tmap), "r"(0), "r"(y),
+                        "r"(smem_u32(mbar + 1 + b))
+                        : "memory");
+                }
+            } else {
+                bulk_g2s(s_buf + b * CHW, bits + cc * kChunk * W, CHW * 4u, mbar + 1 + b);
+            }
         }
     };
     // With one buffer (W >= 12) the next chunk's TMA is issued as soon as the
@@ -203,7 +276,7 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
             flags[h] = 0x4000u;                  // 0x4000: no row (ragged tail), 0x8000: k out of range
             if (row < rows) {
                 uint32_t cuts;
-                s_occ[row] = row_occupancy<W, KEY_ != 0>(buf + row * H, lane, validocc, qfull, lastm, cuts);
+                s_occ[row] = row_occupancy<W, KEY_ != 0, SWZ>(buf + row * H, lane, validocc, qfull, lastm, cuts);
                 const uint32_t ne = __popc(s_occ[row]);
                 // a row with >= k_max non-empty halves (or cuts) has k > k_max
                 flags[h] = (ne < ch.k_max && cuts < ch.k_max) ? 0u : 0x8000u;
@@ -243,13 +316,14 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
                     uint32_t endP = ch.T, OV = 0, cnt = 0;
                     uint64_t S2 = 0;
                     const uint32_t my_s = smem_u32(buf + r * H);
+                    const uint32_t rx = SWZ ? ((r & 7u) << 4) : 0u;   // swizzle of this row's 16-byte chunks
                     uint32_t v = 0, tb = spo_s;      // current half's remaining bits and chain entries (spo + 32 q)
                     auto step = [&]() {
                         // refill (predicated, no branch): next non-empty half when v is exhausted
                         const uint32_t qn = bfind32(occ);
                         const bool need = (v == 0u);
                         if (need) occ ^= 1u << qn;
-                        v = lds32_if(need, my_s + 4u * qn, v);
+                        v = lds32_if(need, SWZ ? (my_s | ((qn << 2) ^ rx)) : my_s + 4u * qn, v);
                         tb = need ? spo_s + (qn << 8) : tb;
                         const uint32_t bt = bfind32(v);
                         v ^= 1u << bt;
@@ -324,26 +398,61 @@ __global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
 // environment variable SPLIT_EVAL_VARIANT=<i> selects another (tuning only).
 struct EvalVariant {
     void* fn;
-    uint32_t W, NW, RPT, NB;
+    uint32_t W, NW, RPT, NB, SWZ;
 };
 
-template <int W, int NW, int RPT, int NB, int KEY = 0>
+template <int W, int NW, int RPT, int NB, int KEY = 0, bool SWZ = false>
 static EvalVariant eval_variant()
 {
-    return EvalVariant{(void*)eval_batch_w_kernel<W, NW, RPT, NB, KEY>, (uint32_t)W, (uint32_t)NW, (uint32_t)RPT,
-                       (uint32_t)NB};
+    return EvalVariant{(void*)eval_batch_w_kernel<W, NW, RPT, NB, KEY, SWZ>, (uint32_t)W, (uint32_t)NW,
+                       (uint32_t)RPT, (uint32_t)NB, SWZ ? 1u : 0u};
 }
 
 static size_t eval_smem_of(const ChainDev& ch, const EvalVariant& v)
 {
     const size_t chunk = (size_t)v.NW * 32 * v.RPT;
-    return (size_t)ch.po_bytes + 32 + chunk * (4 + 2) + 32 * 4 + (size_t)v.NB * chunk * (2 * v.W) * 4;
+    return (size_t)ch.po_bytes + 32 + chunk * (4 + 2) + 32 * 4 + (size_t)v.NB * chunk * (2 * v.W) * 4 +
+           (v.SWZ ? 1024 : 0);
+}
+
+// cuTensorMapEncodeTiled from the driver (the runtime is linked statically; the
+// driver entry point needs no link-time dependency on libcuda)
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_tiled()
+{
+    static EncodeTiledFn fn = [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        return (EncodeTiledFn)p;
+    }();
+    return fn;
+}
+
+// 2-D map over the bitsets viewed as u32 halves: [n_cand rows][32 halves], box of
+// box_rows rows, 128-byte swizzle, zero fill past the last row
+static bool make_row_tmap(CUtensorMap* m, const uint64_t* bits, uint64_t n_cand, uint32_t box_rows)
+{
+    EncodeTiledFn enc = encode_tiled();
+    if (!enc) return false;
+    const cuuint64_t dims[2] = {32, (cuuint64_t)n_cand};
+    const cuuint64_t strides[1] = {128};
+    const cuuint32_t box[2] = {32, box_rows};
+    const cuuint32_t estr[2] = {1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, (void*)bits, dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 template <int W>
 static EvalVariant eval_default()
 {
-    if constexpr (W >= 12) return eval_variant<W, 15, 1, 1>();
+    if constexpr (W == 16) return eval_variant<W, 15, 1, 1, 0, true>();
+    else if constexpr (W >= 12) return eval_variant<W, 15, 1, 1>();
     else if constexpr (W >= 6) return eval_variant<W, 8, 2, 1>();
     else return eval_variant<W, 8, 2, 2>();
 }
@@ -356,6 +465,11 @@ static EvalVariant eval_pick(uint32_t W)
     }();
     if (W == 16 && sel >= 0) {
         switch (sel) {
+        case 100: return eval_variant<16, 15, 1, 1>();            // the round-1 default (bulk copies, no swizzle)
+        case 101: return eval_variant<16, 15, 1, 1, 1, true>();
+        case 102: return eval_variant<16, 16, 1, 1, 0, true>();
+        case 103: return eval_variant<16, 12, 1, 1, 0, true>();
+        case 104: return eval_variant<16, 8, 2, 1, 0, true>();
         case 0: return eval_variant<16, 8, 1, 1>();
         case 1: return eval_variant<16, 7, 2, 1>();
         case 2: return eval_variant<16, 12, 2, 1>();
@@ -386,7 +500,7 @@ static EvalVariant eval_pick(uint32_t W)
     case 10: return eval_default<10>(); case 11: return eval_default<11>(); case 12: return eval_default<12>();
     case 13: return eval_default<13>(); case 14: return eval_default<14>(); case 15: return eval_default<15>();
     case 16: return eval_default<16>();
-    default: return EvalVariant{(void*)eval_batch_kernel, W, (uint32_t)kEvalWarps, 0, 0};
+    default: return EvalVariant{(void*)eval_batch_kernel, W, (uint32_t)kEvalWarps, 0, 0, 0};
     }
 }
 
@@ -394,7 +508,15 @@ cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t
                               int num_sms, uint64_t* launches)
 {
     if (n_cand == 0) return cudaSuccess;
-    const EvalVariant v = eval_pick(ch.W);
+    EvalVariant v = eval_pick(ch.W);
+    alignas(64) CUtensorMap tmap;
+    memset(&tmap, 0, sizeof(tmap));
+    if (v.SWZ) {
+        // tensor maps take int32 row coordinates: larger batches use the bulk-copy kernel
+        const uint32_t chunk = v.NW * 32 * v.RPT, nbox = (chunk + 255) / 256;
+        if (n_cand >= (1ull << 31) || !make_row_tmap(&tmap, bits, n_cand, chunk / nbox))
+            v = eval_variant<16, 15, 1, 1>();
+    }
     const size_t sm = v.RPT ? eval_smem_of(ch, v)
                             : (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
     cudaError_t e = cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
@@ -411,7 +533,7 @@ cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t
     ChainDev c = ch;
     const uint64_t* b = bits;
     double* o = out;
-    void* args[] = {&c, &b, &n_cand, &o};
+    void* args[] = {&c, &b, &n_cand, &o, &tmap};
     e = cudaLaunchKernel(v.fn, dim3((unsigned)grid), dim3(nt), args, sm, st);
     if (launches) ++*launches;
     return e;

@@ -200,7 +200,7 @@ def split_qos_simulate(blocks, arrival, type_id, alpha_milli, policy: int = 1, *
                                                 al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep, n_req,
                                                 arrival.data_ptr(), type_id.data_ptr(), t_ete.data_ptr(),
                                                 viol.data_ptr(), rr.data_ptr(), device, _stream_handle(stream)),
-               "split_qos_simulate_elastic", "split_block_times", "split_heatmap2")
+               "split_qos_simulate_elastic")
         return t_ete, viol, rr
     _check(lib().split_qos_simulate(flat.ctypes.data_as(C.POINTER(C.c_int64)), nb.ctypes.data_as(C.POINTER(C.c_uint32)),
                                     len(blocks), policy, al.ctypes.data_as(C.POINTER(C.c_uint32)), len(al), n_rep,

@@ -69,7 +69,8 @@ def test_c1_exhaustive_eval(S, kind):
     assert got2[0] == -math.inf and _bits_equal(got2[1:], ref[1:])
 
 
-@pytest.mark.parametrize("n", [2, 3, 12, 37, 64, 65, 66, 105, 128, 129, 175, 400, 1024, 2534])
+@pytest.mark.parametrize("n", [2, 3, 12, 37, 64, 65, 66, 105, 128, 129, 175, 400,
+                               961, 993, 1000, 1024, 1025, 2534])   # W = 16 (swizzled K1): every padding shape
 def test_random_batches_and_edges(S, n):
     scale = max(1, n // 64)          # keep (k_max-1) * T'^2 < 2^63 with k_max = n (a0 guard)
     lat, ovh = wl.random_chain(n, 1000 + n, lo=0, hi=200_000 // scale, ovh_hi=30_000 // scale)

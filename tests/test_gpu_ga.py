@@ -243,3 +243,40 @@ def test_k_sweep_eq1_choice(S, name):
     k_star = min(J, key=lambda k: (J[k], k))
     assert 2 < k_star < k_hi                        # the criterion has an interior optimum here
     assert kb == k_star
+
+
+def test_c2_full_length_parity(S):
+    """The bench step itself (C2: n = 175, N = 65,536, E = 1024, s = 4, 500 generations):
+    final population, every fitness bit, the best record and the counters against the
+    oracle GA (about half a minute of one CPU core)."""
+    lat, ovh = wl.chain("resnet50_175")
+    run_both(S, lat, ovh, 500, 1, pop_size=65536, n_elite=1024, tournament_size=4, p_crossover=0.9,
+             p_mutation=0.2, k_min=2, k_max=32)
+
+
+def test_c4_shaped_batched_islands(S):
+    """C4's island model shape (BERT-base chain, W = 7; top-64 migration every 10
+    generations) with 8 islands of 65,536 batched on one GPU, 30 generations: every
+    island bit for bit against the oracle's serial islands."""
+    lat, ovh = wl.chain("bert_base")
+    run_both(S, lat, ovh, 30, 8, pop_size=65536, n_elite=1024, k_min=2, k_max=32, n_islands=8,
+             migration_interval=10, n_migrants=64)
+
+
+def test_comm_layout_checked_at_create(S):
+    """A communicator of world 1 cannot host islands of another layout (advisor: the
+    all-gathers would write past the buffers); the device must match too."""
+    uid = S.split_comm_unique_id()
+    comm = S.split_comm_init(uid, 0, 1, 0)
+    try:
+        lat, ovh = wl.chain("vgg16")
+        for bad in (dict(n_islands=2, islands_per_device=1, island_id=0),
+                    dict(n_islands=2, islands_per_device=1, island_id=1)):
+            with pytest.raises(S.SplitError) as e:
+                S.SplitGA(lat, ovh, comm=comm, pop_size=64, n_elite=2, migration_interval=2, n_migrants=2, **bad)
+            assert e.value.code == S.SPLIT_E_INVAL
+        with S.SplitGA(lat, ovh, comm=comm, pop_size=64, n_elite=2, n_islands=2, islands_per_device=2,
+                       migration_interval=2, n_migrants=2) as h:
+            h.run(3, 1)
+    finally:
+        S.split_comm_destroy(comm)
