@@ -821,8 +821,49 @@ __device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, cons
         row_load(x, popc + (size_t)rx[r] * W, W);
         row_store(x, popn + (size_t)r * W, W);
     }
-    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) fitn[r] = unkey(rk[r]);
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+        fitn[r] = unkey(rk[r]);
+        // the ranked list stays available to the export (top-K = first K) and the migrant merge
+        a.rk_key[(size_t)i * kMaxElite + r] = rk[r];
+        a.rk_idx[(size_t)i * kMaxElite + r] = rx[r];
+    }
     if (threadIdx.x == 0) a.tau[cur * a.I + i] = rk[E - 1];
+}
+
+// ------------------------------------------------------------------------
+// Island exchange blocks (R16, R19): block of global island gi = xch + gi * xstride
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t* xblock(const GaArgs& a, uint32_t gi) { return a.xch + (size_t)gi * a.xstride; }
+__device__ __forceinline__ uint64_t* xrecord(const GaArgs& a, uint32_t gi)
+{
+    return xblock(a, gi) + (size_t)a.K * a.ch.W + a.K;
+}
+
+// leader: island i's record (cached in sm.rec) into its block
+__device__ void pack_record(const GaArgs& a, uint32_t i, const Smem& sm)
+{
+    if (threadIdx.x == 0) {
+        uint64_t* r = xrecord(a, a.island_base + i);
+        const RecCache* rc = sm.rec;
+        r[0] = (uint64_t)__double_as_longlong(rc->valid ? rc->f : -CUDART_INF);
+        r[1] = rc->gen;
+        for (uint32_t w = 0; w < a.ch.W; ++w) r[2 + w] = rc->valid ? rc->bits[w] : ~0ull;
+    }
+}
+
+// leader: export island i's top-K of generation g (ranked list ix[0..K) of slots) -- rows and fitness
+__device__ void export_migrants(const GaArgs& a, uint32_t i, uint32_t g, const uint32_t* ix)
+{
+    const uint32_t W = a.ch.W, cur = g & 1u;
+    const uint64_t* pop = a.pop[cur] + (size_t)i * a.N * W;
+    const double* fit = a.fit[cur] + (size_t)i * a.Ns;
+    uint64_t* blk = xblock(a, a.island_base + i);
+    for (uint32_t j = threadIdx.x; j < a.K * W; j += blockDim.x) {
+        const uint32_t r = j / W, w = j % W;
+        blk[j] = pop[(size_t)ix[r] * W + w];
+    }
+    for (uint32_t r = threadIdx.x; r < a.K; r += blockDim.x)
+        blk[(size_t)a.K * W + r] = (uint64_t)__double_as_longlong(fit[ix[r]]);
 }
 
 // Leader, general path: the radix select already gathered the E best of
@@ -1209,6 +1250,202 @@ __device__ __forceinline__ void precompute_draws(const GaArgs& a, uint32_t i, ui
     }
 }
 
+// sync-point phase stamps (SPLIT_TRACE builds): CTA 0 writes row `row`, slot `slot`
+__device__ __forceinline__ void trace_sync(const GaArgs& a, uint32_t row, uint32_t slot)
+{
+    if (kTrace && a.trace && (a.export_end || row == 15) && blockIdx.x == 0 && threadIdx.x == 0 && row < a.trace_gens)
+        a.trace[row * 16 + slot] = gtimer();
+}
+
+// ------------------------------------------------------------------------
+// Island sync point (R16): the K worst slots of generation g (all CTAs).
+// A strided fitness sample sets, per island, a threshold on the worst key
+// ~fkey(f) that about kWorstCap/2 entries reach; one pass over the islands
+// collects them; the leader sorts the collection (worst order: f asc, index
+// desc) and keeps the first K.  The K worst are all collected whenever at
+// least K entries were (every uncollected entry is better than the
+// threshold), so the result is exact; when a collection holds fewer than K or
+// overflows, every CTA falls back to the radix select.  Islands of at most
+// kWorstSample individuals are sorted whole.
+// ------------------------------------------------------------------------
+template <int WT>
+__device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::grid_group& grid)
+{
+    const uint32_t I = a.I, N = a.N, K = a.K, cur = g & 1u;
+    const bool whole = N <= kWorstSample;
+    if (blockIdx.x < I) {
+        const uint32_t i = blockIdx.x;
+        const double* fit = a.fit[cur] + (size_t)i * a.Ns;
+        const uint32_t S = whole ? N : kWorstSample;
+        const uint32_t P2 = next_pow2(S < 2 ? 2 : S);
+        for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+            if (j < S) {
+                const uint32_t idx = whole ? j : (uint32_t)(((uint64_t)j * N) / S);
+                sm.skey[j] = ~fkey(__ldcg(fit + idx));
+                sm.sidx[j] = ~idx;                      // equal fitness: the larger index is worse
+            } else {
+                sm.skey[j] = 0;
+                sm.sidx[j] = NONE;
+            }
+        }
+        bitonic_desc(sm.skey, sm.sidx, P2);
+        if (whole) {
+            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.sidx[r];
+        } else if (threadIdx.x == 0) {
+            const uint64_t want = (kWorstCap + K) / 2;  // aim between K and the capacity
+            const uint64_t pts = (want * S) / N;       // sample points at or beyond the threshold
+            a.wthr[i] = sm.skey[pts > 0 ? (uint32_t)(pts - 1) : 0u];
+            a.wl_cnt[i] = 0;
+        }
+    }
+    if (whole) return;                                 // uniform across CTAs (N is)
+    trace_sync(a, a.g_end - a.g_begin, 4);
+    grid.sync();
+    const uint64_t total = (uint64_t)I * N;
+    const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t gstride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t e = gtid; e < total; e += gstride) {
+        const uint32_t i = (uint32_t)(e / N), idx = (uint32_t)(e % N);
+        const uint64_t wk = ~fkey(__ldcg(a.fit[cur] + (size_t)i * a.Ns + idx));
+        if (wk >= __ldcg(a.wthr + i)) {
+            const uint32_t pos = atomicAdd(a.wl_cnt + i, 1u);
+            if (pos < kWorstCap) {
+                a.wl_key[(size_t)i * kWorstCap + pos] = wk;
+                a.wl_idx[(size_t)i * kWorstCap + pos] = ~idx;
+            }
+        }
+    }
+    trace_sync(a, a.g_end - a.g_begin, 5);
+    grid.sync();
+    trace_sync(a, a.g_end - a.g_begin, 6);
+    bool ok = true;
+    for (uint32_t i = 0; i < I; ++i) {
+        const uint32_t c = __ldcg(a.wl_cnt + i);
+        ok &= (c >= K && c <= kWorstCap);
+    }
+    if (ok) {
+        if (blockIdx.x < I) {
+            const uint32_t i = blockIdx.x, C = __ldcg(a.wl_cnt + i), P2 = next_pow2(C < 2 ? 2 : C);
+            for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+                sm.skey[j] = j < C ? __ldcg(a.wl_key + (size_t)i * kWorstCap + j) : 0ull;
+                sm.sidx[j] = j < C ? __ldcg(a.wl_idx + (size_t)i * kWorstCap + j) : NONE;
+            }
+            bitonic_desc(sm.skey, sm.sidx, P2);
+            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.sidx[r];
+        }
+    } else {
+        general_select(a, a.fit[cur], K, true, sm, grid);
+        if (blockIdx.x < I) {
+            leader_sort_selected(a, blockIdx.x, K, true, sm);
+            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)blockIdx.x * kMaxElite + r] = sm.sidx[r];
+        }
+    }
+}
+
+// Leader of island i at the head of the segment after sync point g: the K best
+// foreign migrants (f desc, source island asc, rank asc) replace the K worst
+// slots (worst first, R16); the island record takes them in (R19); generation
+// g's ranked elites are merged with them (only K slots changed: no new top-E
+// selection) and placed in slots 0..E-1 of g+1 with the exact threshold.
+template <int WT>
+__device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm)
+{
+    const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I, cur = g & 1u;
+    uint64_t* pop = a.pop[cur] + (size_t)i * N * W;
+    double* fit = a.fit[cur] + (size_t)i * a.Ns;
+    const uint32_t* worst_slot = a.wslot + (size_t)i * kMaxElite;
+    const uint32_t gi = a.island_base + i;
+    const uint32_t nf = (a.I_total - 1) * a.K;
+    const uint32_t P2 = next_pow2(nf < 2 ? 2 : nf);
+    for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
+        if (j < nf) {
+            const uint32_t src = j / a.K, r = j % a.K;
+            const uint32_t gsrc = src < gi ? src : src + 1;   // skip own island
+            sm.skey[j] = fkey(__longlong_as_double((long long)__ldcg(xblock(a, gsrc) + (size_t)a.K * W + r)));
+            sm.sidx[j] = gsrc * a.K + r;
+        } else {
+            sm.skey[j] = 0;
+            sm.sidx[j] = NONE;
+        }
+    }
+    bitonic_desc(sm.skey, sm.sidx, P2);
+    const uint32_t take = a.K < nf ? a.K : nf;
+    for (uint32_t j = threadIdx.x; j < take * W; j += blockDim.x) {
+        const uint32_t r = j / W, w = j % W, e = sm.sidx[r];
+        pop[(size_t)__ldcg(worst_slot + r) * W + w] = __ldcg(xblock(a, e / a.K) + (size_t)(e % a.K) * W + w);
+    }
+    for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) fit[__ldcg(worst_slot + r)] = unkey(sm.skey[r]);
+    __syncthreads();
+    // record update with the received migrants (R19)
+    BestRef v{-CUDART_INF, NONE};
+    for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) {
+        const uint32_t ws = __ldcg(worst_slot + r);
+        const BestRef o{fit[ws], ws};
+        if (better_rec(o.f, o.idx, v.f, v.idx, pop, W)) v = o;
+    }
+    v = block_best(v, pop, W, sm.scratch);
+    if (threadIdx.x == 0 && v.idx != NONE) {
+        bool upd = !a.rec_valid[i];
+        if (!upd) upd = (v.f != a.rec_f[i]) ? (v.f > a.rec_f[i])
+                                             : rows_less(pop + (size_t)v.idx * W, a.rec_bits + (size_t)i * W, W);
+        if (upd) {
+            a.rec_f[i] = v.f;
+            a.rec_gen[i] = g;
+            a.rec_valid[i] = 1;
+            for (uint32_t w = 0; w < W; ++w) a.rec_bits[(size_t)i * W + w] = pop[(size_t)v.idx * W + w];
+        }
+    }
+    if (E == 0) {
+        if (threadIdx.x == 0) a.tau[cur * I + i] = ~0ull;
+        return;
+    }
+    // migrants in ranking order (f desc, slot asc); ranks by binary search against the ranked elites
+    // (disjoint slots: K <= N - E), written to sel_* and placed like any elite set
+    const uint32_t P3 = next_pow2(take < 2 ? 2 : take);
+    for (uint32_t j = threadIdx.x; j < P3; j += blockDim.x) {
+        if (j < take) {
+            sm.sidx[j] = __ldcg(worst_slot + j);       // skey[j] is already that migrant's key
+        } else {
+            sm.skey[j] = 0;
+            sm.sidx[j] = NONE;
+        }
+    }
+    bitonic_desc(sm.skey, sm.sidx, P3);
+    // the ranked elites into shared memory (one round trip) for the binary searches
+    uint64_t* ek = sm.okey;
+    uint32_t* ex = sm.oidx;
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+        ek[r] = __ldcg(a.rk_key + (size_t)i * kMaxElite + r);
+        ex[r] = __ldcg(a.rk_idx + (size_t)i * kMaxElite + r);
+    }
+    __syncthreads();
+    uint64_t* ok = a.sel_key + (size_t)i * kMaxElite;
+    uint32_t* ox = a.sel_idx + (size_t)i * kMaxElite;
+    for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
+        const uint64_t k = ek[r];
+        const uint32_t x = ex[r];
+        uint32_t lo = 0, hi = take;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (comp_gt(sm.skey[mid], sm.sidx[mid], k, x)) lo = mid + 1; else hi = mid;
+        }
+        if (r + lo < E) { ok[r + lo] = k; ox[r + lo] = x; }
+    }
+    for (uint32_t j = threadIdx.x; j < take; j += blockDim.x) {
+        const uint64_t k = sm.skey[j];
+        const uint32_t x = sm.sidx[j];
+        uint32_t lo = 0, hi = E;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (comp_gt(ek[mid], ex[mid], k, x)) lo = mid + 1; else hi = mid;
+        }
+        if (j + lo < E) { ok[j + lo] = k; ox[j + lo] = x; }
+    }
+    __syncthreads();
+    leader_copy_elites<WT>(a, i, g, ok, ox);
+    __syncthreads();
+}
+
 // ------------------------------------------------------------------------
 // The cooperative persistent GA kernel.  CTAs 0..I-1 are island leaders
 // (elite selection, records); the others breed.  One grid barrier per
@@ -1268,78 +1505,7 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
         if (is_leader) {
             rec_load(a, blockIdx.x, sm);
             leader_record<WT>(a, blockIdx.x, 0, 0, sm);
-        }
-        return;
-    }
-
-    if (a.mode == MODE_EXPORT || a.mode == MODE_IMPORT) {
-        const uint32_t g = a.g_begin, cur = g & 1u;
-        const bool worst = a.mode == MODE_IMPORT;
-        general_select(a, a.fit[cur], a.K, worst, sm, grid);
-        if (is_leader) {
-            const uint32_t i = blockIdx.x;
-            leader_sort_selected(a, i, a.K, worst, sm);
-            uint64_t* pop = a.pop[cur] + (size_t)i * N * W;
-            double* fit = a.fit[cur] + (size_t)i * Ns;
-            if (!worst) {
-                // export the island's top-K (rows + fitness) to its slot of the gather buffer
-                const size_t gi = a.island_base + i;
-                for (uint32_t j = threadIdx.x; j < a.K * W; j += blockDim.x) {
-                    const uint32_t r = j / W, w = j % W;
-                    a.mig_bits[(gi * a.K + r) * W + w] = pop[(size_t)sm.sidx[r] * W + w];
-                }
-                for (uint32_t r = threadIdx.x; r < a.K; r += blockDim.x) a.mig_f[gi * a.K + r] = fit[sm.sidx[r]];
-            } else {
-                // worst slots in sidx[0..K); foreign migrants sorted by (f desc, source asc, rank asc)
-                uint32_t* worst_slot = (uint32_t*)sm.ekey;   // K <= kMaxElite u32 fit in ekey
-                for (uint32_t r = threadIdx.x; r < a.K; r += blockDim.x) worst_slot[r] = sm.sidx[r];
-                __syncthreads();
-                const uint32_t gi = a.island_base + i;
-                const uint32_t nf = (a.I_total - 1) * a.K;
-                const uint32_t P2 = next_pow2(nf < 2 ? 2 : nf);
-                for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
-                    if (j < nf) {
-                        const uint32_t src = j / a.K, r = j % a.K;
-                        const uint32_t gsrc = src < gi ? src : src + 1;   // skip own island
-                        const uint32_t e = gsrc * a.K + r;
-                        sm.skey[j] = fkey(a.mig_f[e]);
-                        sm.sidx[j] = e;
-                    } else {
-                        sm.skey[j] = 0;
-                        sm.sidx[j] = NONE;
-                    }
-                }
-                bitonic_desc(sm.skey, sm.sidx, P2);
-                const uint32_t take = a.K < nf ? a.K : nf;
-                for (uint32_t j = threadIdx.x; j < take * W; j += blockDim.x) {
-                    const uint32_t r = j / W, w = j % W;
-                    pop[(size_t)worst_slot[r] * W + w] = a.mig_bits[(size_t)sm.sidx[r] * W + w];
-                }
-                for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) fit[worst_slot[r]] = a.mig_f[sm.sidx[r]];
-                __syncthreads();
-                // record update with the received migrants (R19)
-                BestRef v{-CUDART_INF, NONE};
-                for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) {
-                    const BestRef o{fit[worst_slot[r]], worst_slot[r]};
-                    if (better_rec(o.f, o.idx, v.f, v.idx, pop, W)) v = o;
-                }
-                v = block_best(v, pop, W, sm.scratch);
-                if (threadIdx.x == 0 && v.idx != NONE) {
-                    bool upd = !a.rec_valid[i];
-                    if (!upd) upd = (v.f != a.rec_f[i]) ? (v.f > a.rec_f[i])
-                                                         : rows_less(pop + (size_t)v.idx * W, a.rec_bits + (size_t)i * W, W);
-                    if (upd) {
-                        a.rec_f[i] = v.f;
-                        a.rec_gen[i] = g;
-                        a.rec_valid[i] = 1;
-                        for (uint32_t w = 0; w < W; ++w) a.rec_bits[(size_t)i * W + w] = pop[(size_t)v.idx * W + w];
-                    }
-                }
-                // the children's partial bests of this generation may point at replaced slots
-                for (uint32_t j = threadIdx.x; j < cpi; j += blockDim.x)
-                    a.part_idx[((size_t)cur * I + i) * cpp + j] = NONE;
-                if (threadIdx.x == 0 && i == 0) a.ctl->full = 1;
-            }
+            pack_record(a, blockIdx.x, sm);
         }
         return;
     }
@@ -1347,6 +1513,43 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
     // MODE_RUN: generations [g_begin, g_end).  Candidate lists rotate mod 3:
     // list g%3 holds the candidates of generation g (consumed by leader(g)),
     // breed(g) appends generation g+1's to list (g+1)%3, leader(g) resets (g+2)%3.
+    if (__ldcg(&a.ctl->done)) return;            // islands: the stall rule stopped the run at a sync point
+    if (a.after_import) {
+        // sync point g = g_begin, after the all-gather of the exchange blocks: the global record and
+        // the stall rule (R11, R19) -- decided by CTA 0 from the gathered records, identical on every
+        // rank, followed by every CTA -- then the migrant import (leaders), then breeding
+        const uint32_t g = a.g_begin;
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            double gf = -CUDART_INF;
+            for (uint32_t gi = 0; gi < a.I_total; ++gi)
+                gf = fmax(gf, __longlong_as_double((long long)__ldcg(xrecord(a, gi))));
+            if (gf > a.ctl->gf_improve) {
+                a.ctl->gf_improve = gf;
+                a.ctl->g_last_improve = g;
+            }
+            if (a.stall > 0 && g - a.ctl->g_last_improve >= a.stall) {
+                a.ctl->done = 1;
+                a.ctl->gens_run = g;
+            }
+        }
+        trace_sync(a, 15, 0);
+        grid.sync();
+        trace_sync(a, 15, 1);
+        if (__ldcg(&a.ctl->done)) return;
+        if (is_leader) import_migrants<WT>(a, blockIdx.x, g, sm);
+        trace_sync(a, 15, 2);
+        grid.sync();
+        trace_sync(a, 15, 3);
+    }
+    if (a.init_gstall && blockIdx.x == 0 && threadIdx.x == 0) {
+        // global record of generation 0 from the gathered records (read before any block is rewritten:
+        // leaders pack their records only in the segment's tail, after at least one grid barrier)
+        double gf = -CUDART_INF;
+        for (uint32_t gi = 0; gi < a.I_total; ++gi)
+            gf = fmax(gf, __longlong_as_double((long long)__ldcg(xrecord(a, gi))));
+        a.ctl->gf_improve = gf;
+        a.ctl->g_last_improve = 0;
+    }
     const bool first_full = __ldcg(&a.ctl->full) != 0;
     uint32_t mph = 0;
     ChildDraws pre;
@@ -1376,7 +1579,9 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
         const uint32_t cur = g & 1u, nxt = cur ^ 1u;
         const uint32_t Lb = (g + 1u) % 3u;
         uint32_t tau_par = nxt;               // fast path: worst elite of generation g-1 (lagged)
-        if (g == a.g_begin && first_full && E > 0) {
+        if (g == a.g_begin && a.after_import) {
+            tau_par = cur;                    // the import placed generation g's elites (exact threshold)
+        } else if (g == a.g_begin && first_full && E > 0) {
             // generation 0 or just after migration: exact top-E first, then breed
             general_select(a, a.fit[cur], E, false, sm, grid);
             if (is_leader) {
@@ -1452,10 +1657,43 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
             grid.sync();
         }
     }
-    if (g == a.g_end && is_leader) {
-        // record (and stall) of the last generation of the segment
-        const uint32_t R = __ldcg(a.rc_cnt + (g % 3u) * I + blockIdx.x);
-        leader_record_list<WT>(a, blockIdx.x, g, R, false, sm);
+    if (g == a.g_end) {
+        trace_sync(a, a.g_end - a.g_begin, 0);
+        if (a.export_end && E > 0) {
+            // sync point: generation g's elite step now (record + candidate merge, or the exact radix
+            // path after an overflow); the import merges the migrants into its ranked list
+            if (is_leader) leader_fast<WT>(a, blockIdx.x, g, sm, mph);
+            trace_sync(a, a.g_end - a.g_begin, 1);
+            grid.sync();
+            trace_sync(a, a.g_end - a.g_begin, 2);
+            if (__ldcg(&a.ctl->redo[g & 1u]) == g + 1) {
+                general_select(a, a.fit[g & 1u], E, false, sm, grid);
+                if (is_leader) leader_general<WT>(a, blockIdx.x, g, sm);
+            }
+        } else if (is_leader) {
+            // record (and stall) of the last generation of the segment
+            const uint32_t R = __ldcg(a.rc_cnt + (g % 3u) * I + blockIdx.x);
+            leader_record_list<WT>(a, blockIdx.x, g, R, false, sm);
+        }
+        if (a.export_end) {
+            if (E > 0 && a.K <= E) {
+                if (is_leader) {
+                    __syncthreads();
+                    export_migrants(a, blockIdx.x, g, a.rk_idx + (size_t)blockIdx.x * kMaxElite);   // top-K = first K
+                }
+            } else {
+                // K > E (or E = 0): the island's top-K by the radix select
+                general_select(a, a.fit[g & 1u], a.K, false, sm, grid);
+                if (is_leader) {
+                    leader_sort_selected(a, blockIdx.x, a.K, false, sm);
+                    export_migrants(a, blockIdx.x, g, sm.sidx);
+                }
+            }
+        }
+        trace_sync(a, a.g_end - a.g_begin, 3);
+        if (a.export_end) select_worst<WT>(a, g, sm, grid);
+        trace_sync(a, a.g_end - a.g_begin, 7);
+        if (is_leader) pack_record(a, blockIdx.x, sm);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->gens_run = g;
 }

@@ -164,7 +164,6 @@ struct split_ga_t {
     int64_t* d_stats;
     double* d_statf;
     uint64_t* d_bits1;
-    uint64_t* d_recpack;   // [I_total][W + 2]
     cudaEvent_t ev[4];
     unsigned long long* d_trace;   // SPLIT_TRACE=<csv path>: phase timestamps of the first RUN segment
     uint32_t trace_gens;
@@ -445,7 +444,8 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     a.stall = p.stall_generations;
     a.thr_c = bern_thr(p.p_crossover);
     a.thr_m = bern_thr(p.p_mutation);
-    uint32_t sc = std::max<uint32_t>(pow2_at_least(kCandCap), pow2_at_least(std::max<uint32_t>(a.E, 2)));
+    uint32_t sc = std::max<uint32_t>(pow2_at_least(std::max(kCandCap, std::max(kWorstCap, kWorstSample))),
+                                     pow2_at_least(std::max<uint32_t>(a.E, 2)));
     if (migrate) sc = std::max(sc, pow2_at_least((p.n_islands - 1) * a.K));
     a.sort_cap = sc;
     a.Ns = (a.N + 3u) & ~3u;
@@ -511,14 +511,20 @@ extern "C" int split_ga_create(const int64_t* lat, uint32_t n, const split_ga_pa
     plan.add(&a.rec_bits, (size_t)a.I * h->W);
     plan.add(&a.rec_gen, a.I);
     plan.add(&a.rec_valid, a.I);
-    plan.add(&a.mig_bits, (size_t)a.I_total * std::max<uint32_t>(a.K, 1) * h->W);
-    plan.add(&a.mig_f, (size_t)a.I_total * std::max<uint32_t>(a.K, 1));
+    a.xstride = a.K * h->W + a.K + 2 + h->W;
+    plan.add(&a.xch, (size_t)a.I_total * a.xstride);
+    plan.add(&a.rk_key, (size_t)a.I * kMaxElite);
+    plan.add(&a.rk_idx, (size_t)a.I * kMaxElite);
+    plan.add(&a.wslot, (size_t)a.I * kMaxElite);
+    plan.add(&a.wthr, a.I);
+    plan.add(&a.wl_key, (size_t)a.I * kWorstCap);
+    plan.add(&a.wl_idx, (size_t)a.I * kWorstCap);
+    plan.add(&a.wl_cnt, a.I);
     plan.add(&a.ctl, 1);
     plan.add(&a.gbar, 4);
     plan.add(&h->d_stats, 8);
     plan.add(&h->d_statf, 1);
     plan.add(&h->d_bits1, h->W);
-    plan.add(&h->d_recpack, (size_t)a.I_total * (h->W + 2));
     if (getenv("SPLIT_TRACE")) {
         h->trace_gens = 64;
         plan.add(&h->d_trace, (size_t)h->trace_gens * 16 + kTraceArrGens * 1024);   // + per-CTA arrivals
@@ -691,7 +697,11 @@ extern "C" int split_eval_batch_host(split_ga_t* h, const uint64_t* bits_host, u
 // ------------------------------------------------------------------------
 // a1, a3-a9: the GA driver
 // ------------------------------------------------------------------------
-static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
+struct RunFlags {
+    uint32_t export_end = 0, after_import = 0, init_gstall = 0;
+};
+
+static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1, RunFlags fl = RunFlags{})
 {
     GaArgs a = h->ga;
     if (mode == MODE_RUN) {
@@ -703,6 +713,9 @@ static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1)
     a.trace_gens = h->trace_gens;
     a.g_begin = g0;
     a.g_end = g1;
+    a.export_end = fl.export_end;
+    a.after_import = fl.after_import;
+    a.init_gstall = fl.init_gstall;
     cudaError_t e = launch_ga(a, h->grid, h->stream, &h->stats.launches);
     if (e != cudaSuccess) return fail(SPLIT_E_CUDA, "GA kernel (mode %u): %s", mode, cudaGetErrorString(e));
     return SPLIT_OK;
@@ -716,15 +729,16 @@ static bool rec_better(double fa, const uint64_t* a, double fb, const uint64_t* 
     return false;
 }
 
-// all-gather a device buffer: each rank contributes `bytes` at offset rank*bytes
-static int allgather(split_ga_t* h, void* base, size_t bytes)
+// all-gather the exchange blocks in place: rank r contributes its islands' blocks at offset r * I blocks
+static int allgather_xch(split_ga_t* h)
 {
     SplitComm* c = (SplitComm*)h->p.comm;
-    if (!c) return SPLIT_OK;                 // every island on this device: buffer already complete
+    if (!c) return SPLIT_OK;                 // every island on this device: the blocks are already complete
     NcclApi* api = nccl_api();
     if (!api) return fail(SPLIT_E_NCCL, "NCCL not loadable");
-    const char* src = (const char*)base + (size_t)c->rank * bytes;
-    ncclResult_t r = api->allGather(src, base, bytes, ncclUint8, c->comm, h->stream);
+    const size_t bytes = (size_t)h->ga.I * h->ga.xstride * 8;
+    const char* src = (const char*)h->ga.xch + (size_t)c->rank * bytes;
+    ncclResult_t r = api->allGather(src, h->ga.xch, bytes, ncclUint8, c->comm, h->stream);
     if (r != ncclSuccess) return fail(SPLIT_E_NCCL, "ncclAllGather: %s", api->getErrorString(r));
     return SPLIT_OK;
 }
@@ -735,28 +749,16 @@ struct GlobalRec {
     std::vector<uint64_t> bits;
 };
 
-// gather island records across ranks; returns the global best (R19)
-static int global_record(split_ga_t* h, GlobalRec* best)
+// global best (R19) from the island records in the exchange blocks (host copy)
+static void global_record(split_ga_t* h, const std::vector<uint64_t>& xch, GlobalRec* best)
 {
-    const uint32_t W = h->W, I = h->ga.I, It = h->ga.I_total;
-    const size_t stride = W + 2;
-    // pack local records at this rank's slot: [f bits][gen][W words]
-    uint64_t* slot = h->d_recpack + (size_t)h->ga.island_base * stride;
-    for (uint32_t i = 0; i < I; ++i) {
-        CU(cudaMemcpyAsync(slot + i * stride, h->ga.rec_f + i, 8, cudaMemcpyDeviceToDevice, h->stream));
-        CU(cudaMemcpyAsync(slot + i * stride + 1, h->ga.rec_gen + i, 4, cudaMemcpyDeviceToDevice, h->stream));
-        CU(cudaMemcpyAsync(slot + i * stride + 2, h->ga.rec_bits + (size_t)i * W, W * 8, cudaMemcpyDeviceToDevice, h->stream));
-    }
-    int rc = allgather(h, h->d_recpack, (size_t)I * stride * 8);
-    if (rc) return rc;
-    std::vector<uint64_t> host((size_t)It * stride);
-    CU(cudaMemcpyAsync(host.data(), h->d_recpack, host.size() * 8, cudaMemcpyDeviceToHost, h->stream));
-    CU(cudaStreamSynchronize(h->stream));
+    const uint32_t W = h->W, K = h->ga.K, It = h->ga.I_total;
+    const size_t X = h->ga.xstride;
     bool have = false;
     const uint32_t first = h->p.comm ? 0 : h->ga.island_base;
-    const uint32_t last = h->p.comm ? It : h->ga.island_base + I;
+    const uint32_t last = h->p.comm ? It : h->ga.island_base + h->ga.I;
     for (uint32_t g = first; g < last; ++g) {
-        const uint64_t* e = host.data() + (size_t)g * stride;
+        const uint64_t* e = xch.data() + (size_t)g * X + (size_t)K * W + K;
         double f;
         memcpy(&f, e, 8);
         const uint32_t gen = (uint32_t)(e[1] & 0xFFFFFFFFu);
@@ -769,9 +771,13 @@ static int global_record(split_ga_t* h, GlobalRec* best)
             have = true;
         }
     }
-    return SPLIT_OK;
 }
 
+// Island segments are enqueued back to back with no host synchronisation: at a sync point g
+// (g % M == 0, g < G) the RUN segment ends with the elite step of g, its K worst slots and each
+// island's exchange block (top-K migrants + record); one ncclAllGather moves every block; the
+// next segment's head applies the stall rule (ctl->done stops every later launch), places the
+// foreign migrants and merges them into g's elites, then breeds.
 extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, split_best_t* best_out)
 {
     if (!h || !best_out) return fail(SPLIT_E_INVAL, "split_ga_run: NULL argument");
@@ -792,61 +798,44 @@ extern "C" int split_ga_run(split_ga_t* h, uint32_t generations, uint64_t seed, 
     int rc = run_kernel(h, MODE_INIT, 0, 0);
     if (rc) return rc;
     CU(cudaEventRecord(h->ev[1], h->stream));
-    uint32_t gens_run = 0;
     const uint32_t M = h->p.migration_interval;
-    if (single || M == 0) {
+    const bool islands = !single && M > 0;
+    if (!islands) {
         if (generations > 0) {
             rc = run_kernel(h, MODE_RUN, 0, generations);
             if (rc) return rc;
         }
-        Ctl ctl;
-        CU(cudaMemcpyAsync(&ctl, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, h->stream));
-        CU(cudaStreamSynchronize(h->stream));
-        gens_run = generations > 0 ? ctl.gens_run : 0;
-        h->stats.general_selects = ctl.n_general;
-        h->stats.fast_selects = ctl.n_fast;
     } else {
-        GlobalRec gr;
-        rc = global_record(h, &gr);
+        rc = allgather_xch(h);                        // generation-0 records: the global stall baseline
         if (rc) return rc;
-        double f_improve = gr.f;
-        uint32_t last_improve = 0;
         uint32_t g = 0;
         while (g < generations) {
             const uint32_t g1 = std::min<uint32_t>((g / M + 1) * M, generations);
-            rc = run_kernel(h, MODE_RUN, g, g1);
+            RunFlags fl;
+            fl.export_end = (g1 % M == 0 && g1 < generations) ? 1u : 0u;
+            fl.after_import = g > 0 ? 1u : 0u;
+            fl.init_gstall = g == 0 ? 1u : 0u;
+            rc = run_kernel(h, MODE_RUN, g, g1, fl);
+            if (rc) return rc;
+            if (!fl.export_end) break;
+            rc = allgather_xch(h);                    // the next segment's head imports from the blocks
             if (rc) return rc;
             g = g1;
-            Ctl ctl;
-            CU(cudaMemcpyAsync(&ctl, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, h->stream));
-            CU(cudaStreamSynchronize(h->stream));
-            h->stats.general_selects += ctl.n_general;
-            h->stats.fast_selects += ctl.n_fast;
-            if (g % M != 0) break;   // g == generations, not a sync point
-            rc = global_record(h, &gr);
-            if (rc) return rc;
-            if (gr.f > f_improve) {
-                f_improve = gr.f;
-                last_improve = g;
-            }
-            if (h->p.stall_generations > 0 && g - last_improve >= h->p.stall_generations) break;
-            if (g < generations) {
-                rc = run_kernel(h, MODE_EXPORT, g, g);
-                if (rc) return rc;
-                rc = allgather(h, a.mig_bits, (size_t)a.I * a.K * h->W * 8);
-                if (rc) return rc;
-                rc = allgather(h, a.mig_f, (size_t)a.I * a.K * 8);
-                if (rc) return rc;
-                rc = run_kernel(h, MODE_IMPORT, g, g);
-                if (rc) return rc;
-            }
         }
-        gens_run = g;
     }
     CU(cudaEventRecord(h->ev[2], h->stream));
-    GlobalRec best;
-    rc = global_record(h, &best);
+    rc = allgather_xch(h);                            // final records (the last launch packed them)
     if (rc) return rc;
+    Ctl ctl;
+    std::vector<uint64_t> xh((size_t)a.I_total * a.xstride);
+    CU(cudaMemcpyAsync(&ctl, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaMemcpyAsync(xh.data(), a.xch, xh.size() * 8, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    const uint32_t gens_run = generations > 0 ? ctl.gens_run : 0;
+    h->stats.general_selects = ctl.n_general;
+    h->stats.fast_selects = ctl.n_fast;
+    GlobalRec best;
+    global_record(h, xh, &best);
     // statistics of the best split
     CU(cudaMemcpyAsync(h->d_bits1, best.bits.data(), h->W * 8, cudaMemcpyHostToDevice, h->stream));
     CU(launch_eval_stats(h->ch, h->d_bits1, h->d_stats, h->d_statf, h->stream));

@@ -15,7 +15,9 @@ constexpr uint32_t kTraceArrGens = 8;       // SPLIT_TRACE: generations whose pe
 constexpr uint32_t kBlock = 512;            // threads per CTA of the GA kernel (one CTA per SM)
 
 enum Tag : uint32_t { TAG_INIT = 1, TAG_SELECT = 2, TAG_XOVER = 3, TAG_MUTATE = 4, TAG_REPAIR = 5 };
-enum Mode : uint32_t { MODE_INIT = 0, MODE_RUN = 1, MODE_EXPORT = 2, MODE_IMPORT = 3 };
+enum Mode : uint32_t { MODE_INIT = 0, MODE_RUN = 1 };
+constexpr uint32_t kWorstCap = 2048;        // worst-slot candidates collected per island at a sync point
+constexpr uint32_t kWorstSample = 2048;     // fitness sample that sets the collection threshold
 
 // device-resident control block (one per handle)
 struct Ctl {
@@ -26,6 +28,9 @@ struct Ctl {
     double f_improve;       // record fitness at the last improvement
     uint32_t n_general, n_fast;
     uint32_t redo[2];       // redo[g&1] == g+1: a leader's candidate list overflowed in generation g
+    double gf_improve;      // islands: global record at the last strict improvement (sync points, R11)
+    uint32_t g_last_improve;
+    uint32_t pad;
 };
 
 // Chain staged for the kernels: P[0..n] (u32, exclusive prefix of the latencies)
@@ -76,8 +81,20 @@ struct GaArgs {
     uint64_t* rec_bits;                // [I][W]
     uint32_t* rec_gen;                 // [I]
     uint32_t* rec_valid;               // [I]
-    uint64_t* mig_bits;                // [I_total][K][W]
-    double* mig_f;                     // [I_total][K]
+    // exchange blocks, one per GLOBAL island (all-gathered in one NCCL call at a sync point):
+    // [K][W] migrant rows | [K] migrant fitness (f64 bits) | record: f64 bits, generation, [W] bits
+    uint64_t* xch;
+    uint32_t xstride;                  // words per block: K W + K + 2 + W
+    uint32_t export_end;               // RUN: the segment ends at a sync point: elites, export, record
+    uint32_t after_import;             // RUN: generation g_begin's elites were placed by the import
+    uint32_t init_gstall;              // RUN: set the global stall state from the gathered gen-0 records
+    uint64_t* rk_key;                  // [I][kMaxElite] ranked elites of the last elite step (f keys)
+    uint32_t* rk_idx;                  //   and their slots
+    uint32_t* wslot;                   // [I][kMaxElite] the K worst slots (worst first) at the sync point
+    uint64_t* wthr;                    // [I] collection threshold on the worst key ~fkey(f)
+    uint64_t* wl_key;                  // [I][kWorstCap] collected (worst key, ~slot) candidates
+    uint32_t* wl_idx;
+    uint32_t* wl_cnt;                  // [I]
     uint32_t* rc_cnt;                  // [3][I] record-candidate lists (children that beat a
     uint32_t* rc_idx[3];               //        snapshot of the island record), rotation as cand_*
     double* snap_f;                    // [2][I] record snapshots (parity g&1), read by breed(g+1)

@@ -36,6 +36,11 @@ if __name__ == "__main__":
     uid = S.split_comm_unique_id()
     comm = S.split_comm_init(uid, 0, 1, 0)
     G = 500
+    if len(sys.argv) == 3:                      # one configuration, one run (for ncu launch lists)
+        t, _ = run(int(sys.argv[1]), int(sys.argv[2]), G, reps=1, comm=comm)
+        print(f"I={sys.argv[1]} M={sys.argv[2]} {t:.2f} ms")
+        S.split_comm_destroy(comm)
+        sys.exit(0)
     for I in (1, 8):
         base, _ = run(I, 0, G, comm=None if I == 1 else comm)
         print(f"I={I} M=0   {base:8.2f} ms  {G / base * 1e3:9.0f} gens/s", flush=True)
