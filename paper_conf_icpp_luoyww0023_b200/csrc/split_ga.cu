@@ -469,6 +469,7 @@ struct Smem {
     uint64_t* ekey;       // [kMaxElite]
     uint64_t* okey;       // [kMaxElite] merged elites (fast path)
     uint32_t* oidx;
+    uint32_t* tsel;       // [kMaxElite] in-CTA selection output (sync points)
     RecCache* rec;        // leader: island record + stall state, cached for the whole launch
     double* pf;           // [cpi_pad] staged partial bests (leader)
     uint32_t* pi;
@@ -498,6 +499,7 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take((size_t)kMaxElite * 8 + 16); if (s) s->ekey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 8); if (s) s->okey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 4); if (s) s->oidx = (uint32_t*)p;
+    p = take((size_t)kMaxElite * 4); if (s) s->tsel = (uint32_t*)p;
     p = take(sizeof(RecCache) + 8 * (size_t)a.ch.W); if (s) s->rec = (RecCache*)p;
     p = take((size_t)a.cpi_pad * 8); if (s) s->pf = (double*)p;
     p = take(((size_t)a.cpi_pad + 4) * 4); if (s) s->pi = (uint32_t*)p;
@@ -643,6 +645,114 @@ __device__ void general_select(const GaArgs& a, const double* fit, uint32_t Ksel
     if (blockIdx.x == 0) {
         for (uint32_t j = threadIdx.x; j < 3 * I * 256; j += blockDim.x) a.ghist[j] = 0;
     }
+}
+
+// ------------------------------------------------------------------------
+// In-CTA selection (one leader CTA, all its threads): the k largest of n
+// (key, idx) entries in shared memory under the ranking order of comp_gt
+// (key desc, idx asc), by an MSB radix select over the 96-bit composite
+// (key, ~idx) -- a few passes of a 256-bin shared histogram, starting below
+// the key bytes every entry shares; no sort of the n entries (an in-CTA
+// bitonic sort of 2048 entries costs ~29 us on B200,
+// tools/microbench_bitonic.cu; a one-warp select was slower still: its
+// histogram atomics serialise) -- then the k selected are ordered by rank
+// counting into ok/ox[0..k).  hist: 256 words, st: one SelState, counter:
+// one word, tk/tx: >= k scratch; all in shared memory; k <= 1024.
+// ------------------------------------------------------------------------
+__device__ void cta_select_sorted(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t k, uint32_t* hist,
+                                  SelState* st, uint32_t* counter, uint64_t* tk, uint32_t* tx, uint64_t* ok,
+                                  uint32_t* ox)
+{
+    // leading bytes of the key that every entry shares need no pass: the select starts below them
+    if (threadIdx.x == 0) { hist[0] = 0; hist[1] = 0; *counter = 0; }
+    __syncthreads();
+    const uint64_t k0 = n ? key[0] : 0ull;
+    uint64_t diff = 0;
+    for (uint32_t j = threadIdx.x; j < n; j += blockDim.x) diff |= key[j] ^ k0;
+#pragma unroll
+    for (int off = 16; off; off >>= 1) diff |= __shfl_xor_sync(0xFFFFFFFFu, diff, off);
+    if ((threadIdx.x & 31u) == 0 && diff) {
+        atomicOr(hist, (uint32_t)(diff >> 32));
+        atomicOr(hist + 1, (uint32_t)diff);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const uint64_t dall = ((uint64_t)hist[0] << 32) | hist[1];
+        const uint32_t d0 = dall ? (uint32_t)__clzll((long long)dall) / 8u : 8u;   // 0..8 common bytes
+        st->ph = d0 == 0 ? 0ull : (d0 >= 8 ? k0 : (k0 >> (64 - 8 * d0)));
+        st->pl = 0;
+        st->d = d0;
+        st->need = k;
+        st->done = (k >= n) || (k == 0);
+    }
+    __syncthreads();
+    while (!st->done) {
+        for (uint32_t j = threadIdx.x; j < 256; j += blockDim.x) hist[j] = 0;
+        __syncthreads();
+        const SelState s = *st;
+        for (uint32_t j = threadIdx.x; j < n; j += blockDim.x) {
+            const uint64_t hi = key[j];
+            const uint32_t lo = ~idx[j];
+            if (sel_match(hi, lo, s)) atomicAdd(&hist[sel_digit(hi, lo, s.d)], 1u);
+        }
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            const uint32_t lane = threadIdx.x;
+            uint32_t c[8], sum = 0;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) { c[q] = hist[255 - 8 * lane - q]; sum += c[q]; }
+            uint32_t incl = sum;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, incl, off);
+                if (lane >= (uint32_t)off) incl += o;
+            }
+            const uint32_t excl = incl - sum;
+            const bool mine = excl < s.need && incl >= s.need;
+            const int src = __ffs(__ballot_sync(0xFFFFFFFFu, mine)) - 1;
+            uint32_t bin = 0, cnt = 0, before = 0;
+            if (mine) {
+                uint32_t acc = excl;
+                for (int q = 0; q < 8; ++q) {
+                    if (acc + c[q] >= s.need) { bin = 255 - 8 * lane - q; cnt = c[q]; before = acc; break; }
+                    acc += c[q];
+                }
+            }
+            bin = __shfl_sync(0xFFFFFFFFu, bin, src);
+            cnt = __shfl_sync(0xFFFFFFFFu, cnt, src);
+            before = __shfl_sync(0xFFFFFFFFu, before, src);
+            if (lane == 0) {
+                SelState t = s;
+                t.need -= before;
+                if (t.d < 8) t.ph = (t.ph << 8) | bin;
+                else t.pl = (t.pl << 8) | bin;
+                t.d += 1;
+                if (cnt == t.need || t.d == 12) t.done = 1;
+                *st = t;
+            }
+        }
+        __syncthreads();
+    }
+    // the selected entries (exactly min(k, n)) to tk/tx, then ordered by rank counting
+    const SelState s = *st;
+    const bool all = k >= n;
+    for (uint32_t j = threadIdx.x; j < n; j += blockDim.x) {
+        if (all || sel_selected(key[j], ~idx[j], s)) {
+            const uint32_t p = atomicAdd(counter, 1u);
+            if (p < k) { tk[p] = key[j]; tx[p] = idx[j]; }
+        }
+    }
+    __syncthreads();
+    const uint32_t m = min(*counter, k);
+    for (uint32_t j = threadIdx.x; j < m; j += blockDim.x) {
+        const uint64_t kj = tk[j];
+        const uint32_t xj = tx[j];
+        uint32_t r = 0;
+        for (uint32_t q = 0; q < m; ++q) r += comp_gt(tk[q], tx[q], kj, xj) ? 1u : 0u;
+        ok[r] = kj;
+        ox[r] = xj;
+    }
+    __syncthreads();
 }
 
 // Leader CTA: sort the general-select output of island i in smem (ranking
@@ -1277,44 +1387,72 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
         const uint32_t i = blockIdx.x;
         const double* fit = a.fit[cur] + (size_t)i * a.Ns;
         const uint32_t S = whole ? N : kWorstSample;
-        const uint32_t P2 = next_pow2(S < 2 ? 2 : S);
-        for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
-            if (j < S) {
-                const uint32_t idx = whole ? j : (uint32_t)(((uint64_t)j * N) / S);
-                sm.skey[j] = ~fkey(__ldcg(fit + idx));
-                sm.sidx[j] = ~idx;                      // equal fitness: the larger index is worse
-            } else {
-                sm.skey[j] = 0;
-                sm.sidx[j] = NONE;
-            }
+        for (uint32_t j = threadIdx.x; j < S; j += blockDim.x) {
+            const uint32_t idx = whole ? j : (uint32_t)(((uint64_t)j * N) / S);
+            sm.skey[j] = ~fkey(__ldcg(fit + idx));
+            sm.sidx[j] = ~idx;                          // equal fitness: the larger index is worse
         }
-        bitonic_desc(sm.skey, sm.sidx, P2);
+        __syncthreads();
         if (whole) {
-            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.sidx[r];
-        } else if (threadIdx.x == 0) {
+            cta_select_sorted(sm.skey, sm.sidx, S, K, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.tsel[r];
+        } else {
             const uint64_t want = (kWorstCap + K) / 2;  // aim between K and the capacity
-            const uint64_t pts = (want * S) / N;       // sample points at or beyond the threshold
-            a.wthr[i] = sm.skey[pts > 0 ? (uint32_t)(pts - 1) : 0u];
-            a.wl_cnt[i] = 0;
+            uint64_t pts = (want * S) / N;             // sample points at or beyond the threshold
+            pts = pts < 1 ? 1 : pts;
+            cta_select_sorted(sm.skey, sm.sidx, S, (uint32_t)pts, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx,
+                              sm.ekey, sm.tsel);
+            if (threadIdx.x == 0) {
+                a.wthr[i] = sm.ekey[pts - 1];           // the smallest selected key: >= pts sample points reach it
+                a.wl_cnt[i] = 0;
+            }
         }
     }
     if (whole) return;                                 // uniform across CTAs (N is)
     trace_sync(a, a.g_end - a.g_begin, 4);
     grid.sync();
-    const uint64_t total = (uint64_t)I * N;
-    const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const uint64_t gstride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t e = gtid; e < total; e += gstride) {
-        const uint32_t i = (uint32_t)(e / N), idx = (uint32_t)(e % N);
-        const uint64_t wk = ~fkey(__ldcg(a.fit[cur] + (size_t)i * a.Ns + idx));
-        if (wk >= __ldcg(a.wthr + i)) {
-            const uint32_t pos = atomicAdd(a.wl_cnt + i, 1u);
-            if (pos < kWorstCap) {
-                a.wl_key[(size_t)i * kWorstCap + pos] = wk;
-                a.wl_idx[(size_t)i * kWorstCap + pos] = ~idx;
+    // one pass over the islands (I N < 2^32, checked at create): each CTA counts its entries per
+    // island in shared memory, reserves one range per island with a single global atomic, then
+    // writes them (the count and write passes see the same entries)
+    const uint32_t total = I * N, gtid = blockIdx.x * blockDim.x + threadIdx.x, gstride = gridDim.x * blockDim.x;
+    uint32_t* lcnt = sm.hist;                          // [I] counts, [I] bases at +16
+    uint64_t* lthr = (uint64_t*)(sm.hist + 32);        // [I] thresholds
+    if (threadIdx.x < 32) lcnt[threadIdx.x] = 0;
+    if (threadIdx.x < I) lthr[threadIdx.x] = __ldcg(a.wthr + threadIdx.x);
+    __syncthreads();
+    // eight loads in flight per thread and pass (the pass is latency-bound, not bandwidth-bound)
+    constexpr uint32_t U = 8;
+    auto scan = [&](bool write) {
+        for (uint32_t e0 = gtid; e0 < total; e0 += U * gstride) {
+            uint64_t wk[U];
+#pragma unroll
+            for (uint32_t u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * gstride;
+                const uint32_t i = e / N;
+                wk[u] = e < total ? ~fkey(__ldcg(a.fit[cur] + (size_t)i * a.Ns + (e - i * N))) : 0ull;
+            }
+#pragma unroll
+            for (uint32_t u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * gstride;
+                const uint32_t i = e / N;
+                if (e < total && wk[u] >= lthr[i]) {
+                    const uint32_t p = atomicAdd(lcnt + i, 1u);
+                    if (write && lcnt[16 + i] + p < kWorstCap) {
+                        a.wl_key[(size_t)i * kWorstCap + lcnt[16 + i] + p] = wk[u];
+                        a.wl_idx[(size_t)i * kWorstCap + lcnt[16 + i] + p] = ~(e - i * N);
+                    }
+                }
             }
         }
+    };
+    scan(false);
+    __syncthreads();
+    if (threadIdx.x < I) {
+        lcnt[16 + threadIdx.x] = lcnt[threadIdx.x] ? atomicAdd(a.wl_cnt + threadIdx.x, lcnt[threadIdx.x]) : 0u;
+        lcnt[threadIdx.x] = 0;
     }
+    __syncthreads();
+    scan(true);
     trace_sync(a, a.g_end - a.g_begin, 5);
     grid.sync();
     trace_sync(a, a.g_end - a.g_begin, 6);
@@ -1325,13 +1463,14 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
     }
     if (ok) {
         if (blockIdx.x < I) {
-            const uint32_t i = blockIdx.x, C = __ldcg(a.wl_cnt + i), P2 = next_pow2(C < 2 ? 2 : C);
-            for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
-                sm.skey[j] = j < C ? __ldcg(a.wl_key + (size_t)i * kWorstCap + j) : 0ull;
-                sm.sidx[j] = j < C ? __ldcg(a.wl_idx + (size_t)i * kWorstCap + j) : NONE;
+            const uint32_t i = blockIdx.x, C = __ldcg(a.wl_cnt + i);
+            for (uint32_t j = threadIdx.x; j < C; j += blockDim.x) {
+                sm.skey[j] = __ldcg(a.wl_key + (size_t)i * kWorstCap + j);
+                sm.sidx[j] = __ldcg(a.wl_idx + (size_t)i * kWorstCap + j);
             }
-            bitonic_desc(sm.skey, sm.sidx, P2);
-            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.sidx[r];
+            __syncthreads();
+            cta_select_sorted(sm.skey, sm.sidx, C, K, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+            for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.tsel[r];
         }
     } else {
         general_select(a, a.fit[cur], K, true, sm, grid);
@@ -1356,25 +1495,21 @@ __device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const S
     const uint32_t* worst_slot = a.wslot + (size_t)i * kMaxElite;
     const uint32_t gi = a.island_base + i;
     const uint32_t nf = (a.I_total - 1) * a.K;
-    const uint32_t P2 = next_pow2(nf < 2 ? 2 : nf);
-    for (uint32_t j = threadIdx.x; j < P2; j += blockDim.x) {
-        if (j < nf) {
-            const uint32_t src = j / a.K, r = j % a.K;
-            const uint32_t gsrc = src < gi ? src : src + 1;   // skip own island
-            sm.skey[j] = fkey(__longlong_as_double((long long)__ldcg(xblock(a, gsrc) + (size_t)a.K * W + r)));
-            sm.sidx[j] = gsrc * a.K + r;
-        } else {
-            sm.skey[j] = 0;
-            sm.sidx[j] = NONE;
-        }
+    for (uint32_t j = threadIdx.x; j < nf; j += blockDim.x) {
+        const uint32_t src = j / a.K, r = j % a.K;
+        const uint32_t gsrc = src < gi ? src : src + 1;   // skip own island
+        sm.skey[j] = fkey(__longlong_as_double((long long)__ldcg(xblock(a, gsrc) + (size_t)a.K * W + r)));
+        sm.sidx[j] = gsrc * a.K + r;                        // ascending in (source island, rank)
     }
-    bitonic_desc(sm.skey, sm.sidx, P2);
+    __syncthreads();
     const uint32_t take = a.K < nf ? a.K : nf;
+    // the K best foreign migrants in order (f desc, source asc, rank asc) -> ekey/tsel[0..take)
+    cta_select_sorted(sm.skey, sm.sidx, nf, take, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
     for (uint32_t j = threadIdx.x; j < take * W; j += blockDim.x) {
-        const uint32_t r = j / W, w = j % W, e = sm.sidx[r];
+        const uint32_t r = j / W, w = j % W, e = sm.tsel[r];
         pop[(size_t)__ldcg(worst_slot + r) * W + w] = __ldcg(xblock(a, e / a.K) + (size_t)(e % a.K) * W + w);
     }
-    for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) fit[__ldcg(worst_slot + r)] = unkey(sm.skey[r]);
+    for (uint32_t r = threadIdx.x; r < take; r += blockDim.x) fit[__ldcg(worst_slot + r)] = unkey(sm.ekey[r]);
     __syncthreads();
     // record update with the received migrants (R19)
     BestRef v{-CUDART_INF, NONE};
@@ -1399,18 +1534,20 @@ __device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const S
         if (threadIdx.x == 0) a.tau[cur * I + i] = ~0ull;
         return;
     }
-    // migrants in ranking order (f desc, slot asc); ranks by binary search against the ranked elites
-    // (disjoint slots: K <= N - E), written to sel_* and placed like any elite set
-    const uint32_t P3 = next_pow2(take < 2 ? 2 : take);
-    for (uint32_t j = threadIdx.x; j < P3; j += blockDim.x) {
-        if (j < take) {
-            sm.sidx[j] = __ldcg(worst_slot + j);       // skey[j] is already that migrant's key
-        } else {
-            sm.skey[j] = 0;
-            sm.sidx[j] = NONE;
-        }
+    // migrants in ranking order (f desc, slot asc) by rank counting into skey/sidx[0..take); ranks by
+    // binary search against the ranked elites (disjoint slots: K <= N - E), written to sel_* and
+    // placed like any elite set
+    for (uint32_t j = threadIdx.x; j < take; j += blockDim.x) sm.tsel[j] = __ldcg(worst_slot + j);
+    __syncthreads();
+    for (uint32_t j = threadIdx.x; j < take; j += blockDim.x) {
+        const uint64_t kj = sm.ekey[j];
+        const uint32_t xj = sm.tsel[j];
+        uint32_t r = 0;
+        for (uint32_t q = 0; q < take; ++q) r += comp_gt(sm.ekey[q], sm.tsel[q], kj, xj) ? 1u : 0u;
+        sm.skey[r] = kj;
+        sm.sidx[r] = xj;
     }
-    bitonic_desc(sm.skey, sm.sidx, P3);
+    __syncthreads();
     // the ranked elites into shared memory (one round trip) for the binary searches
     uint64_t* ek = sm.okey;
     uint32_t* ex = sm.oidx;
@@ -1556,7 +1693,10 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
     bool have_pre = false;
     double fpre[4];                   // prefetched fitness of the first tournament (s <= 4)
     bool have_fpre = false;
-    unsigned int bar_target = 0;      // generation barrier counter (zeroed by the host per launch)
+    // generation barrier: a monotonic counter; this launch starts where the previous one left it
+    // (ctl->gbar_base is written only after the last arrival of a launch, so every CTA reads the
+    // same base before any arrival of this one)
+    unsigned int bar_target = __ldcg(&a.ctl->gbar_base);
     BestRow<WT> snap;
     snap.f = -CUDART_INF;         // first phase of a launch: no filter (all children compared)
     snap.idx = 0;
@@ -1695,7 +1835,10 @@ __global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
         trace_sync(a, a.g_end - a.g_begin, 7);
         if (is_leader) pack_record(a, blockIdx.x, sm);
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->gens_run = g;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.ctl->gens_run = g;
+        a.ctl->gbar_base = bar_target;
+    }
 }
 
 // ------------------------------------------------------------------------

@@ -704,10 +704,6 @@ struct RunFlags {
 static int run_kernel(split_ga_t* h, uint32_t mode, uint32_t g0, uint32_t g1, RunFlags fl = RunFlags{})
 {
     GaArgs a = h->ga;
-    if (mode == MODE_RUN) {
-        cudaError_t me = cudaMemsetAsync(a.gbar, 0, 16, h->stream);
-        if (me != cudaSuccess) return fail(SPLIT_E_CUDA, "barrier reset: %s", cudaGetErrorString(me));
-    }
     a.mode = mode;
     a.trace = (mode == MODE_RUN) ? h->d_trace : nullptr;
     a.trace_gens = h->trace_gens;

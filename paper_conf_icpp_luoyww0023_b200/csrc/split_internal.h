@@ -30,7 +30,7 @@ struct Ctl {
     uint32_t redo[2];       // redo[g&1] == g+1: a leader's candidate list overflowed in generation g
     double gf_improve;      // islands: global record at the last strict improvement (sync points, R11)
     uint32_t g_last_improve;
-    uint32_t pad;
+    uint32_t gbar_base;     // generation-barrier count reached by the last RUN launch (monotonic)
 };
 
 // Chain staged for the kernels: P[0..n] (u32, exclusive prefix of the latencies)
