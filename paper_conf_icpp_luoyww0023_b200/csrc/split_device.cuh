@@ -66,6 +66,14 @@ __device__ __forceinline__ uint32_t bfind32(uint32_t x)
     return r;
 }
 
+// (1 << b) - 1: the bits below position b (one BMSK)
+__device__ __forceinline__ uint32_t bmsk32(uint32_t b)
+{
+    uint32_t r;
+    asm("bmsk.clamp.b32 %0, 0, %1;" : "=r"(r) : "r"(b));
+    return r;
+}
+
 // ------------------------------------------------------------------------
 // dexp: exp by the fixed operation sequence of DESIGN.md R5'' (Cody-Waite
 // reduction, degree-13 Taylor polynomial in Horner form, RN(1/i!)).

@@ -190,6 +190,53 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
     return occ;
 }
 
+// The walk of one row (the a2 core): visit its cuts from the last one down, one loop
+// iteration per cut -- a predicated refill from the occupancy mask `occ` when the
+// current half is exhausted, one FLO for the cut -- summing the exact integer
+// statistics from the staged {P[p+1], ovh[p]} pairs (spo_s), then the FP64 tail of
+// Eq. 2.  my_s: shared address of the row's 32-bit halves; SWZ: 128-byte swizzle
+// by (r & 7).
+template <bool SWZ>
+__device__ __forceinline__ double walk_row(const ChainDev& ch, uint32_t occ, uint32_t my_s, uint32_t r, uint32_t spo_s)
+{
+    uint32_t endP = ch.T, OV = 0, cnt = 0;
+    uint64_t S2 = 0;
+    const uint32_t rx = SWZ ? ((r & 7u) << 4) : 0u;   // swizzle of this row's 16-byte chunks
+    uint32_t v = 0, tb = spo_s;      // current half's remaining bits and chain entries (spo + 32 q)
+    auto step = [&]() {
+        // refill (predicated, no branch): next non-empty half when v is exhausted -- clear its
+        // occupancy bit (the highest: mask below it), load it, point tb at its chain entries;
+        // then take v's highest cut the same way
+        const uint32_t qn = bfind32(occ);
+        const bool need = (v == 0u);
+        occ = need ? (occ & bmsk32(qn)) : occ;
+        v = lds32_if(need, SWZ ? (my_s | ((qn << 2) ^ rx)) : my_s + 4u * qn, v);
+        tb = need ? spo_s + (qn << 8) : tb;
+        const uint32_t bt = bfind32(v);
+        v &= bmsk32(bt);                 // clears bit bt, the highest set
+        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+        const uint2 e = lds64(tb + 8u * bt);
+        const uint32_t tj = endP - e.x + e.y;
+        S2 += (uint64_t)tj * tj;
+        OV += e.y;
+        endP = e.x;
+    };
+    // unrolled by two (no register moves between iterations)
+    while (v | occ) {
+        step();
+        cnt += 1;
+        if (!(v | occ)) break;
+        step();
+        cnt += 1;
+    }
+    const uint32_t k = cnt + 1;
+    if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
+    S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
+    const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
+    const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
+    return eq2(k, V, OV, ch);
+}
+
 // SWZ (W = 16): every chunk -- the ragged last one included (rows past n_cand
 // arrive zero-filled) -- is one or two tensor TMA copies (box: 32 halves x
 // CHUNK/nbox rows, 128-byte swizzle) described by `tmap`; the chunk buffer is
@@ -204,25 +251,23 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
     constexpr uint32_t H = Cfg::H, CHW = Cfg::CHW, NB = Cfg::NB, NT = Cfg::NT, kChunk = Cfg::CHUNK;
     constexpr uint32_t kBoxes = (kChunk + 255u) / 256u, kBoxRows = kChunk / kBoxes;
     static_assert(!SWZ || (W == 16 && kBoxRows * kBoxes == kChunk && NT % 8 == 0), "swizzled chunk geometry");
-    extern __shared__ __align__(16) uint8_t smem[];
+    // the chunk buffers first: the dynamic window starts 1024-byte aligned, as the 128-byte swizzle needs
+    extern __shared__ __align__(1024) uint8_t smem_k1[];
+    uint8_t* smem = smem_k1;
+    uint32_t* s_buf = (uint32_t*)smem;                   // [NB][CHW]
     // staged chain: po[p] = {P[p+1], ovh[p]} for cut positions p in [0, n-2]
-    const uint2* spo = (const uint2*)smem;
-    uint64_t* mbar = (uint64_t*)(smem + ch.po_bytes);   // [0] chain, [1], [2] chunk buffers, [3] pad
+    const uint2* spo = (const uint2*)(smem + (size_t)NB * CHW * 4u);
+    uint64_t* mbar = (uint64_t*)((const uint8_t*)spo + ch.po_bytes);   // [0] chain, [1], [2] chunk buffers, [3] pad
     uint32_t* s_occ = (uint32_t*)(mbar + 4);             // [kChunk] occupancy mask of each row
     uint32_t* s_hist = s_occ + kChunk;                   // [32] histogram of the sort keys
     uint16_t* s_perm = (uint16_t*)(s_hist + 32);         // [kChunk] sorted order | flags
-    uint32_t* s_buf = (uint32_t*)(s_perm + kChunk);      // [NB][CHW] (16-byte aligned)
-    if constexpr (SWZ) {
-        const uint32_t a = smem_u32(s_buf);
-        s_buf = (uint32_t*)((uint8_t*)s_buf + (((a + 1023u) & ~1023u) - a));
-    }
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     if (tid == 0) {
         mbar_init(mbar + 1, 1);
         mbar_init(mbar + 2, 1);
     }
     if (tid < 32) s_hist[tid] = 0;
-    stage_bulk(smem, ch.po, ch.po_bytes, mbar);           // includes a __syncthreads
+    stage_bulk((void*)spo, ch.po, ch.po_bytes, mbar);     // includes a __syncthreads
     const uint32_t npos = ch.n - 1, qfull = npos >> 5;
     const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
     const uint32_t validocc = (qfull >= 32u) ? ~0u : ((1u << qfull) - 1u);   // halves wholly inside [0, n-2]
@@ -309,48 +354,8 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
             const uint32_t pe = s_perm[32u * grp + lane];
             const uint32_t r = pe & 0x3FFFu;
             if (pe & 0x4000u) continue;
-            double f = -CUDART_INF;
-            if (!(pe & 0x8000u)) {
-                {
-                    uint32_t occ = s_occ[r];
-                    uint32_t endP = ch.T, OV = 0, cnt = 0;
-                    uint64_t S2 = 0;
-                    const uint32_t my_s = smem_u32(buf + r * H);
-                    const uint32_t rx = SWZ ? ((r & 7u) << 4) : 0u;   // swizzle of this row's 16-byte chunks
-                    uint32_t v = 0, tb = spo_s;      // current half's remaining bits and chain entries (spo + 32 q)
-                    auto step = [&]() {
-                        // refill (predicated, no branch): next non-empty half when v is exhausted
-                        const uint32_t qn = bfind32(occ);
-                        const bool need = (v == 0u);
-                        if (need) occ ^= 1u << qn;
-                        v = lds32_if(need, SWZ ? (my_s | ((qn << 2) ^ rx)) : my_s + 4u * qn, v);
-                        tb = need ? spo_s + (qn << 8) : tb;
-                        const uint32_t bt = bfind32(v);
-                        v ^= 1u << bt;
-                        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
-                        const uint2 e = lds64(tb + 8u * bt);
-                        const uint32_t tj = endP - e.x + e.y;
-                        S2 += (uint64_t)tj * tj;
-                        OV += e.y;
-                        endP = e.x;
-                    };
-                    // unrolled by two (no register moves between iterations)
-                    while (v | occ) {
-                        step();
-                        cnt += 1;
-                        if (!(v | occ)) break;
-                        step();
-                        cnt += 1;
-                    }
-                    const uint32_t k = cnt + 1;
-                    if (k >= ch.k_min && k <= ch.k_max) {
-                        S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
-                        const uint64_t S1 = (uint64_t)ch.T + OV;     // sum of block times = T + overheads
-                        const int64_t V = (int64_t)((uint64_t)k * S2 - S1 * S1);
-                        f = eq2(k, V, OV, ch);
-                    }
-                }
-            }
+            const double f = (pe & 0x8000u) ? -CUDART_INF
+                                            : walk_row<SWZ>(ch, s_occ[r], smem_u32(buf + r * H), r, spo_s);
             __stcs(out + row0 + r, f);
         }
         __syncthreads();                         // buffer b, s_occ, s_perm released
@@ -411,8 +416,7 @@ static EvalVariant eval_variant()
 static size_t eval_smem_of(const ChainDev& ch, const EvalVariant& v)
 {
     const size_t chunk = (size_t)v.NW * 32 * v.RPT;
-    return (size_t)ch.po_bytes + 32 + chunk * (4 + 2) + 32 * 4 + (size_t)v.NB * chunk * (2 * v.W) * 4 +
-           (v.SWZ ? 1024 : 0);
+    return (size_t)ch.po_bytes + 32 + chunk * (4 + 2) + 32 * 4 + (size_t)v.NB * chunk * (2 * v.W) * 4;
 }
 
 // cuTensorMapEncodeTiled from the driver (the runtime is linked statically; the
@@ -451,7 +455,7 @@ static bool make_row_tmap(CUtensorMap* m, const uint64_t* bits, uint64_t n_cand,
 template <int W>
 static EvalVariant eval_default()
 {
-    if constexpr (W == 16) return eval_variant<W, 15, 1, 1, 0, true>();
+    if constexpr (W == 16) return eval_variant<W, 11, 1, 1, 0, true>();   // 4 CTAs x 11 warps per SM
     else if constexpr (W >= 12) return eval_variant<W, 15, 1, 1>();
     else if constexpr (W >= 6) return eval_variant<W, 8, 2, 1>();
     else return eval_variant<W, 8, 2, 2>();
@@ -470,6 +474,11 @@ static EvalVariant eval_pick(uint32_t W)
         case 102: return eval_variant<16, 16, 1, 1, 0, true>();
         case 103: return eval_variant<16, 12, 1, 1, 0, true>();
         case 104: return eval_variant<16, 8, 2, 1, 0, true>();
+        case 110: return eval_variant<16, 10, 1, 1, 0, true>();
+        case 111: return eval_variant<16, 11, 1, 1, 0, true>();
+        case 113: return eval_variant<16, 13, 1, 1, 0, true>();
+        case 114: return eval_variant<16, 14, 1, 1, 0, true>();
+        case 116: return eval_variant<16, 16, 1, 1, 0, true>();
         case 0: return eval_variant<16, 8, 1, 1>();
         case 1: return eval_variant<16, 7, 2, 1>();
         case 2: return eval_variant<16, 12, 2, 1>();
