@@ -140,55 +140,106 @@ class ClockSampler:
 
 
 def ga_bytes_per_generation(N: int, E: int, W: int, s: int) -> int:
-    """Algorithmic HBM bytes of one generation: per child one parent row
-    read (pairs read two rows for two children), one child row and one f64 written, s
-    f64 tournament gathers; the elite step reads N f64 and copies E rows + f64."""
-    return (N - E) * (16 * W + 8 + 8 * s) + 8 * N + 2 * E * (8 * W + 8)
+    """Algorithmic HBM bytes of one generation (16W + 16 + 8s B per child --
+    a parent row read and the child row written (pairs read two rows for two children), the
+    child's f64 written and one elite-threshold key read, s f64 tournament gathers -- plus
+    8N for the elite step's fitness read and 2E(8W + 8) for the elite copy)."""
+    return (N - E) * (16 * W + 16 + 8 * s) + 8 * N + 2 * E * (8 * W + 8)
+
+
+def _latency_floor() -> dict | None:
+    """Measured floor of one GA generation (profiles/latency_floor.json: grid barrier plus
+    two dependent L2 round trips, tools/microbench_gridbar.cu on this pool's B200)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "latency_floor.json")) as f:
+            return json.load(f)
+    except Exception:
+        return None
 
 
 def eval_bytes_per_candidate(W: int) -> int:
     return 8 * W + 8
 
 
-def cpu_baseline_oracle(generations: int) -> dict:
+def _cpu_model() -> str:
+    try:
+        txt = open("/proc/cpuinfo").read()
+        return txt.split("model name")[1].split("\n")[0].strip(": \t") if "model name" in txt else "unknown"
+    except Exception:
+        return "unknown"
+
+
+class _OneCore:
+    """Pin this process to one host core for a timed oracle call (taskset -c <core>), then restore."""
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = min(self.prev)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.prev)
+
+
+def _timed_ga(chain, generations, **kw):
     import oracle
     from paper_conf_icpp_luoyww0023_b200 import workloads as wl
-    lat, ovh = wl.chain(C2["chain"])
+    lat, ovh = wl.c1_chain() if chain == "c1" else wl.chain(chain)
+    with _OneCore() as oc:
+        t0 = time.perf_counter()
+        r = oracle.ga_run(lat, ovh, generations, 1, **kw)
+        dt = time.perf_counter() - t0
+    return r, dt, oc.core
+
+
+def cpu_baseline_oracle(generations: int) -> dict:
+    """SURVEY §8(d) CPU plan, the oracle as it stands (plain C, single-threaded), pinned to one
+    host core: the headline GA on C2 (bounded sample), plus the GA on C1 and on a C4 island
+    (first 3 generations), and its fitness loop on C5 and C4 rows on one core and on all cores."""
     kw = {k: C2[k] for k in ("pop_size", "n_elite", "tournament_size", "p_crossover", "p_mutation", "k_min", "k_max")}
-    t0 = time.perf_counter()
-    r = oracle.ga_run(lat, ovh, generations, 1, **kw)
-    dt = time.perf_counter() - t0
-    return {"value": r["evaluations"] / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"oracle GA (plain C, 1 thread) on C2: N=65536, {generations} generations "
-                      f"({r['evaluations']} evals) in {dt:.2f} s",
-            "gens_per_s": generations / dt}
+    r, dt, core = _timed_ga(C2["chain"], generations, **kw)
+    out = {"value": r["evaluations"] / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "cpu": _cpu_model(),
+           "pinned_core": core,
+           "sample": f"oracle GA (plain C, 1 thread pinned to core {core}) on C2: N=65536, {generations} "
+                     f"generations ({r['evaluations']} evals) in {dt:.2f} s",
+           "gens_per_s": generations / dt}
+    r1, dt1, _ = _timed_ga("c1", 50, pop_size=256, n_elite=4, k_min=2, k_max=12)
+    out["ga_c1"] = {"evals_per_s": r1["evaluations"] / dt1, "gens_per_s": 50 / dt1, "cores": 1,
+                    "sample": f"C1 (n=12, N=256, 50 generations) in {dt1 * 1e3:.1f} ms"}
+    r4, dt4, _ = _timed_ga("bert_base", 3, pop_size=1 << 20, n_elite=1024, k_min=2, k_max=32)
+    out["ga_c4_first3"] = {"evals_per_s": r4["evaluations"] / dt4, "gens_per_s": 3 / dt4, "cores": 1,
+                           "sample": f"one C4 island (bert_base n=400, N=1,048,576), generation 0 + 3 generations "
+                                     f"({r4['evaluations']} evals) in {dt4:.2f} s"}
+    for name, chain, n_c in (("eval_c5", "synthetic_1024", 1 << 18), ("eval_c4", "bert_base", 1 << 19)):
+        with _OneCore():
+            t = _oracle_eval_shard((n_c, 999, chain))
+        out[name + "_1core"] = {"evals_per_s": n_c / t, "cores": 1, "sample": f"{n_c} {chain} rows in {t:.2f} s"}
+    return out
 
 
 def _oracle_eval_shard(args):
     import oracle
     from paper_conf_icpp_luoyww0023_b200 import workloads as wl
-    n_cand, seed = args
-    lat, ovh = wl.chain("synthetic_1024")
+    n_cand, seed, chain = args
+    lat, ovh = wl.chain(chain)
     pop = wl.uniform_k_population_fast(len(lat), n_cand, seed=seed)
     t0 = time.perf_counter()
     oracle.fitness_batch(lat, ovh, pop, 2, 32)
     return time.perf_counter() - t0
 
 
-def cpu_eval_all_cores(n_per_core: int = 1 << 18) -> dict:
+def cpu_eval_all_cores(chain: str = "synthetic_1024", n_per_core: int = 1 << 18) -> dict:
     """The oracle's fitness (plain C, single-threaded) as P independent processes on disjoint
-    shards of C5 candidates, P = the host cores this process may use."""
+    shards of C5 (or C4) candidates, P = the host cores this process may use."""
     import multiprocessing as mp
     P = len(os.sched_getaffinity(0))
     ctx = mp.get_context("spawn")
     with ctx.Pool(P) as pool:
-        ts = pool.map(_oracle_eval_shard, [(n_per_core, 1000 + i) for i in range(P)])
+        ts = pool.map(_oracle_eval_shard, [(n_per_core, 1000 + i, chain) for i in range(P)])
     wall = max(ts)                                   # oracle time of the slowest process
-    cpu = open("/proc/cpuinfo").read().split("model name")[1].split("\n")[0].strip(": \t") \
-        if os.path.exists("/proc/cpuinfo") and "model name" in open("/proc/cpuinfo").read() else "unknown"
     return {"value": P * n_per_core / wall, "unit": UNIT, "cores": P, "kind": "oracle",
-            "sample": f"oracle fitness (C5 rows, n = 1024) in {P} processes x {n_per_core} candidates; "
-                      f"slowest process {wall:.2f} s of oracle time", "cpu": cpu}
+            "sample": f"oracle fitness ({chain} rows) in {P} processes x {n_per_core} candidates; "
+                      f"slowest process {wall:.2f} s of oracle time", "cpu": _cpu_model()}
 
 
 def run_reference(args):
@@ -313,17 +364,26 @@ def main():
     gen_bytes = ga_bytes_per_generation(C2["pop_size"], C2["n_elite"], W, C2["tournament_size"])
     loop_avg_ms = sum(loop_ms) / len(loop_ms)
     achieved_gbs = gen_bytes * G / (loop_avg_ms / 1000.0) / 1e9
+    us_gen = 1000.0 * loop_avg_ms / G
+    floor = _latency_floor()
     roofline = {"bound": "hbm", "kernel": "ga_kernel (RUN segment: all generations of a step)",
                 "achieved": achieved_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved_gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
                 "traffic": _profile_traffic("ga_kernel_per_launch"),
                 "algorithmic_bytes_per_generation": gen_bytes,
                 "launch_ms_avg": loop_avg_ms, "share_of_step": loop_avg_ms / (t_max_ms / args.steps),
+                "binding_roof": {
+                    "bound": "latency", "us_per_generation": us_gen,
+                    "floor_us": floor["grid_barrier_plus_2_dependent_l2_us"] if floor else None,
+                    "frac": (floor["grid_barrier_plus_2_dependent_l2_us"] / us_gen) if floor else None,
+                    "floor": "one grid barrier + two dependent L2 round trips per generation, measured on this "
+                             "pool's B200 (profiles/latency_floor.json, tools/microbench_gridbar.cu)"},
                 "note": ("C2's 1.7 MB working set is L2-resident (ncu DRAM traffic per 500-generation launch is "
-                         "the 'traffic' field): the kernel is bound by per-generation latency (two dependent L2 "
-                         "round trips, the fused eval and one grid barrier per generation), not by HBM; the same "
-                         "kernel's HBM regime is 'ga_hbm_regime', the HBM-bound K1 is 'eval_batch' "
-                         "(profiles/r01_notes.md)")}
+                         "the 'traffic' field), so the HBM fraction is not the binding roof: a generation is a "
+                         "grid barrier, dependent L2 round trips (tournament gathers, parent rows), breeding and "
+                         "the fused eval; 'binding_roof' compares it with the measured barrier + L2 floor.  The "
+                         "HBM-bound kernel is K1 ('eval_roofline'); the GA kernel's HBM regime is "
+                         "'ga_hbm_regime'")}
 
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -334,6 +394,7 @@ def main():
         "elite_select_paths": {"radix_general": n_general, "candidate_merge": n_fast},
         "best": {"fitness": best["fitness"], "k": best["k"], "generation_found": best["generation_found"]},
         "roofline": roofline,
+        "eval_roofline": None,          # K1 split_eval_batch at C5 (the north-star's >= 60 % target), filled below
     }
 
     # e2e through the public API with host buffers: set_chain (H2D of the chain) + run + best (D2H)
@@ -389,6 +450,11 @@ def main():
         ms_avg = sum(ms) / len(ms)
         bpc = eval_bytes_per_candidate(W5)
         gbs = bpc * C5_EVAL_N / (ms_avg / 1000.0) / 1e9
+        out["eval_roofline"] = {"kernel": "eval_batch_w_kernel (K1, split_eval_batch)", "bound": "hbm",
+                                "frac": gbs / peaks["hbm_gbs"], "achieved": gbs, "peak": peaks["hbm_gbs"],
+                                "unit": "GB/s", "traffic": _profile_traffic("eval_batch_kernel_c5"),
+                                "algorithmic": f"{eval_bytes_per_candidate(W5)} B/candidate x 2^24",
+                                "evals_per_s": C5_EVAL_N / (ms_avg / 1000.0)}
         out["eval_batch"] = {
             "workload": "C5: synthetic 1024-op chain (W=16), N=2^24 candidates, k ~ U[2,32]",
             "evals_per_s": C5_EVAL_N / (ms_avg / 1000.0), "ms_per_launch": ms_avg,
@@ -495,6 +561,36 @@ def main():
             "evals_per_s": ev4 / (t4 / 1000.0), "ms_per_step": t4 / len(c4ms),
             "gens_per_s": 200 / ((t4 / len(c4ms)) / 1000.0), "n_gpus": world, "scaling": "weak"}
 
+    # island sync points (a9 over the device-side loop): 8 islands of C2 size batched on this GPU with a
+    # 1-rank NCCL communicator, top-64 migration every 10 generations vs no migration; the difference per
+    # sync point is the exchange's cost (export + all-gather + import), with no host synchronisation
+    if not args.no_c4 and world == 1:
+        sync_comm = S.split_comm_init(S.split_comm_unique_id(), 0, 1, local)
+        try:
+            res = {}
+            for M in (0, 10):
+                ikw = dict(pop_size=65536, n_elite=1024, k_min=2, k_max=32, n_islands=8, islands_per_device=8,
+                           migration_interval=M, n_migrants=64 if M else 0)
+                with S.SplitGA(lat, ovh, device=local, stream=stream, comm=sync_comm if M else None, **ikw) as hi:
+                    hi.run(G, 7)
+                    ims = []
+                    for i in range(3):
+                        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        s0.record(stream)
+                        hi.run(G, 8 + i)
+                        s1.record(stream)
+                        torch.cuda.synchronize()
+                        ims.append(s0.elapsed_time(s1))
+                res[M] = statistics.median(ims)
+            syncs = G // 10 - 1
+            out["island_sync"] = {
+                "workload": f"8 islands x 65,536 (C2 chain) on one GPU, {G} generations, top-64 every 10 "
+                            "generations through a 1-rank NCCL communicator vs no migration",
+                "ms_no_migration": res[0], "ms_migration": res[10], "gens_rate_ratio": res[0] / res[10],
+                "us_per_sync_point": 1000.0 * (res[10] - res[0]) / syncs}
+        finally:
+            S.split_comm_destroy(sync_comm)
+
     # f2 QoS simulator: Table 2's heaviest scenario (lambda = 110 ms, 1000 requests) over the
     # paper-five chains split into 4 blocks by the GA, Algorithm 1 vs FIFO, 65,536 replicas
     if not args.no_qos:
@@ -586,7 +682,8 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline_oracle(CPU_SAMPLE_GENERATIONS)
         try:
-            out["cpu_baseline"]["eval_all_cores"] = cpu_eval_all_cores()
+            out["cpu_baseline"]["eval_all_cores"] = cpu_eval_all_cores("synthetic_1024")
+            out["cpu_baseline"]["eval_c4_all_cores"] = cpu_eval_all_cores("bert_base", 1 << 19)
         except Exception as e:                      # reported baseline only; never fails the run
             out["cpu_baseline"]["eval_all_cores"] = {"unavailable": repr(e)[:200]}
     out["paper_context"] = ("PAPER.md profiles 'over 20,000 candidates' offline on a Jetson Nano at ~1 s per "

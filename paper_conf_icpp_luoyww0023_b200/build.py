@@ -46,6 +46,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     os.makedirs(OBJ_DIR, exist_ok=True)
     extra = ["-DSPLIT_TRACE_BUILD"] if os.environ.get("SPLIT_TRACE_BUILD") else []
+    if os.environ.get("SPLIT_GA_MIN_BLOCKS"):            # A/B builds of the GA kernel's occupancy
+        extra.append(f"-DSPLIT_GA_MIN_BLOCKS={int(os.environ['SPLIT_GA_MIN_BLOCKS'])}")
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
     dep_t = _newest_dep()
     procs = []

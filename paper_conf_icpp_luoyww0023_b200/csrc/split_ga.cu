@@ -1589,8 +1589,11 @@ __device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const S
 // generation: leader(g) runs concurrently with breed(g) because breed(g)
 // needs only generation g and a lagged candidate threshold.
 // ------------------------------------------------------------------------
+#ifndef SPLIT_GA_MIN_BLOCKS
+#define SPLIT_GA_MIN_BLOCKS 1
+#endif
 template <int WT>
-__global__ void __launch_bounds__(kBlock, 1) ga_kernel(GaArgs a)
+__global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs a)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     Smem sm;
@@ -1865,7 +1868,7 @@ static void* ga_pick(uint32_t W)
 int ga_max_blocks_per_sm(uint32_t W)
 {
     (void)W;
-    return 1;
+    return SPLIT_GA_MIN_BLOCKS;
 }
 
 int ga_grid(const GaArgs& a, int num_sms, cudaError_t* err)

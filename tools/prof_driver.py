@@ -37,9 +37,10 @@ def main(what: str, reps: int = 3, gens: int = 500):
             S.split_qos_simulate(blocks, da, dt, [1000 * a for a in range(2, 21)], 2 if kw else 1, **kw)
         torch.cuda.synchronize()
         return
-    elif what == "ga_big":
+    elif what in ("ga_big", "ga_1m"):
         lat, ovh = wl.chain("bert_base")
-        h = S.SplitGA(lat, ovh, pop_size=1 << 22, n_elite=1024, k_min=2, k_max=32, stream=st)
+        h = S.SplitGA(lat, ovh, pop_size=(1 << 22) if what == "ga_big" else (1 << 20), n_elite=1024, k_min=2, k_max=32,
+                      stream=st)
         for i in range(reps):
             h.run(gens, i)
     else:
