@@ -918,7 +918,8 @@ __device__ void leader_record_list(const GaArgs& a, uint32_t i, uint32_t g, uint
 // Copy the ranked elites (keys rk, indices rx into generation g) to slots
 // 0..E-1 of generation g+1 (R18) and publish the worst elite's key.
 template <int WT>
-__device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, const uint64_t* rk, const uint32_t* rx)
+__device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, const uint64_t* rk, const uint32_t* rx,
+                                   bool keep_ranked = false)
 {
     const uint32_t W = a.ch.W, N = a.N, E = a.E;
     const uint32_t cur = g & 1u, nxt = cur ^ 1u;
@@ -933,9 +934,11 @@ __device__ void leader_copy_elites(const GaArgs& a, uint32_t i, uint32_t g, cons
     }
     for (uint32_t r = threadIdx.x; r < E; r += blockDim.x) {
         fitn[r] = unkey(rk[r]);
-        // the ranked list stays available to the export (top-K = first K) and the migrant merge
-        a.rk_key[(size_t)i * kMaxElite + r] = rk[r];
-        a.rk_idx[(size_t)i * kMaxElite + r] = rx[r];
+        if (keep_ranked) {
+            // sync point: the ranked list stays available to the export (top-K = first K) and the migrant merge
+            a.rk_key[(size_t)i * kMaxElite + r] = rk[r];
+            a.rk_idx[(size_t)i * kMaxElite + r] = rx[r];
+        }
     }
     if (threadIdx.x == 0) a.tau[cur * a.I + i] = rk[E - 1];
 }
@@ -979,10 +982,10 @@ __device__ void export_migrants(const GaArgs& a, uint32_t i, uint32_t g, const u
 // Leader, general path: the radix select already gathered the E best of
 // generation g; sort them and place them.
 template <int WT>
-__device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm)
+__device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm, bool keep_ranked = false)
 {
     leader_sort_selected(a, i, a.E, false, sm);
-    leader_copy_elites<WT>(a, i, g, sm.skey, sm.sidx);
+    leader_copy_elites<WT>(a, i, g, sm.skey, sm.sidx, keep_ranked);
     __syncthreads();
 }
 
@@ -994,7 +997,8 @@ __device__ void leader_general(const GaArgs& a, uint32_t i, uint32_t g, const Sm
 // overflowed, the leader only stamps ctl->redo[g&1] and every CTA runs the
 // general path after the barrier.
 template <int WT>
-__device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm, uint32_t& mph)
+__device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem& sm, uint32_t& mph,
+                            bool keep_ranked = false)
 {
     const uint32_t Ns = a.Ns, E = a.E, I = a.I, cpi = a.cpi, cpp = a.cpi_pad;
     const uint32_t cur = g & 1u, Lc = g % 3u, Lr = (g + 2u) % 3u;
@@ -1130,7 +1134,7 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
         if (rank < E) { sm.okey[rank] = k; sm.oidx[rank] = sm.sidx[j]; }
     }
     __syncthreads();
-    leader_copy_elites<WT>(a, i, g, sm.okey, sm.oidx);
+    leader_copy_elites<WT>(a, i, g, sm.okey, sm.oidx, keep_ranked);
     if (threadIdx.x == 0 && i == 0) a.ctl->n_fast = ++sm.misc[8];
     trace_mark(a, g, 3);
 }
@@ -1579,7 +1583,7 @@ __device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const S
         if (j + lo < E) { ok[j + lo] = k; ox[j + lo] = x; }
     }
     __syncthreads();
-    leader_copy_elites<WT>(a, i, g, ok, ox);
+    leader_copy_elites<WT>(a, i, g, ok, ox, false);
     __syncthreads();
 }
 
@@ -1805,13 +1809,13 @@ __global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs 
         if (a.export_end && E > 0) {
             // sync point: generation g's elite step now (record + candidate merge, or the exact radix
             // path after an overflow); the import merges the migrants into its ranked list
-            if (is_leader) leader_fast<WT>(a, blockIdx.x, g, sm, mph);
+            if (is_leader) leader_fast<WT>(a, blockIdx.x, g, sm, mph, true);
             trace_sync(a, a.g_end - a.g_begin, 1);
             grid.sync();
             trace_sync(a, a.g_end - a.g_begin, 2);
             if (__ldcg(&a.ctl->redo[g & 1u]) == g + 1) {
                 general_select(a, a.fit[g & 1u], E, false, sm, grid);
-                if (is_leader) leader_general<WT>(a, blockIdx.x, g, sm);
+                if (is_leader) leader_general<WT>(a, blockIdx.x, g, sm, true);
             }
         } else if (is_leader) {
             // record (and stall) of the last generation of the segment

@@ -13,7 +13,8 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
-PROF = os.path.join(ROOT, "profiles")
+PROF = os.environ.get("SPLIT_PROF_OUT") or os.path.join(ROOT, "profiles")   # gpurun_out/ on the GPU box
+REPS = os.environ.get("SPLIT_NCU_DIR") or OUT                                # where the .ncu-rep files are
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__warps_active.avg.pct_of_peak_sustained_active",
@@ -86,10 +87,14 @@ def main(tag):
     traffic = {}
     for name, rep, per in (("ga_kernel", "prof_ga.ncu-rep", "launch (one RUN segment = 500 generations of C2)"),
                            ("eval_batch_kernel", "prof_eval.ncu-rep", "launch (C5, 2^24 candidates)"),
+                           ("ga_kernel, 1M island", "prof_ga_1m.ncu-rep",
+                            "launch (C4 island: bert_base n=400, N=1,048,576, 20 generations from generation 0)"),
+                           ("ga_kernel, 4M island", "prof_ga_4m.ncu-rep",
+                            "launch (HBM regime: bert_base, N=4,194,304, 20 generations from generation 0)"),
                            ("qos_kernel", "prof_qos.ncu-rep", "launch (f2: 65,536 replicas x 1000 requests)"),
                            ("qos_kernel, f4 elastic", "prof_qos_el.ncu-rep",
                             "launch (f4: the same workload, d_max = 3, s_max = 2)")):
-        path = os.path.join(OUT, rep)
+        path = os.path.join(REPS, rep)
         if not os.path.exists(path):
             continue
         m = ncu_raw(path)
