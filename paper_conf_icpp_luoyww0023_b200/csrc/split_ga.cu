@@ -499,12 +499,12 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     p = take((size_t)kMaxElite * 8 + 16); if (s) s->ekey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 8); if (s) s->okey = (uint64_t*)p;
     p = take((size_t)kMaxElite * 4); if (s) s->oidx = (uint32_t*)p;
-    p = take((size_t)kMaxElite * 4); if (s) s->tsel = (uint32_t*)p;
     p = take(sizeof(RecCache) + 8 * (size_t)a.ch.W); if (s) s->rec = (RecCache*)p;
     p = take((size_t)a.cpi_pad * 8); if (s) s->pf = (double*)p;
     p = take(((size_t)a.cpi_pad + 4) * 4); if (s) s->pi = (uint32_t*)p;
     p = take(a.stage_bits ? (size_t)a.cpi_pad * a.ch.W * 8 : 16); if (s) s->pb = (uint64_t*)p;
     p = take((a.ch.W > 4 && a.ch.W <= 16) ? (size_t)kBlock * (2 * a.ch.W + 1) * 4 : 16); if (s) s->rows = (uint32_t*)p;
+    p = take((size_t)kMaxElite * 4); if (s) s->tsel = (uint32_t*)p;
     return off;
 }
 
