@@ -189,8 +189,9 @@ int split_block_times(const int64_t* latencies_ns, const int64_t* cut_overhead_n
  *   rr_out       device double [n_rep][2]: sum of t_ete/Ext and of its square,
  *                added in request order
  * Synchronous.  SPLIT_E_INVAL on bad host arguments; SPLIT_E_RANGE when a
- * replica has unordered arrivals / a bad type id or more than 32 pending
- * requests (an overloaded system: its results are then undefined). */
+ * replica has unordered arrivals / a bad type id, or more than 160 pending
+ * requests (a batch where some replica exceeds 32 is re-run with a 160-entry
+ * queue, more slowly; every output is rewritten). */
 int split_qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint32_t n_types, uint32_t policy,
                        const uint32_t* alpha_milli, uint32_t n_alpha, uint64_t n_rep, uint32_t n_req,
                        const int64_t* arrival_ns, const uint32_t* type_id, int64_t* t_ete_out,

@@ -1251,7 +1251,7 @@ static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint
     a.rr = rr_out;
     a.d_max = d_max;
     a.s_max = s_max;
-    if (qos_smem_bytes(a) > 227 * 1024) return fail(SPLIT_E_INVAL, "split_qos_simulate: model tables too large");
+    if (qos_smem_bytes(a, kQosQueueBig) > 227 * 1024) return fail(SPLIT_E_INVAL, "split_qos_simulate: model tables too large");
     // stream-ordered scratch (no device-wide synchronisation in cudaFree)
     uint32_t* d_tab = nullptr;
     CU(cudaMallocAsync((void**)&d_tab, tab.size() * 4, st));
@@ -1268,12 +1268,20 @@ static int qos_simulate(const int64_t* blocks_ns, const uint32_t* n_blocks, uint
     a.uns = a.blk_ns + blk.size();
     a.ref = a.uns + uns.size();
     a.err = d_tab + tab.size() - 1;
-    CU(launch_qos(a, st));
+    CU(launch_qos(a, st, kQosQueue));
     uint32_t err = 0;
     CU(cudaMemcpyAsync(&err, a.err, 4, cudaMemcpyDeviceToHost, st));
     CU(cudaStreamSynchronize(st));
+    if (err == 2) {
+        // some replica held more than kQosQueue pending requests (an overloaded system): the whole batch
+        // again with the large queue (fewer replicas per SM; every output is rewritten)
+        CU(cudaMemsetAsync(a.err, 0, 4, st));
+        CU(launch_qos(a, st, kQosQueueBig));
+        CU(cudaMemcpyAsync(&err, a.err, 4, cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+    }
     if (err == 1) return fail(SPLIT_E_RANGE, "split_qos_simulate: arrivals not non-decreasing / negative, or type id >= n_types");
-    if (err == 2) return fail(SPLIT_E_RANGE, "split_qos_simulate: more than %u pending requests (overloaded)", kQosQueue);
+    if (err == 2) return fail(SPLIT_E_RANGE, "split_qos_simulate: more than %u pending requests (overloaded)", kQosQueueBig);
     return SPLIT_OK;
 }
 

@@ -129,7 +129,8 @@ size_t exh_smem_bytes(const ExhArgs& a);
 int exh_blocks_per_sm(const ExhArgs& a);
 // f2 QoS simulator (split_qos.cu)
 constexpr uint32_t kQosThreads = 64;    // replicas per CTA (one per thread): 7 CTAs per SM fit 65,536 replicas in one wave
-constexpr uint32_t kQosQueue = 32;      // pending requests a replica may hold
+constexpr uint32_t kQosQueue = 32;      // pending requests a replica may hold (fast form)
+constexpr uint32_t kQosQueueBig = 160;  // the re-run after an overflow (overloaded systems)
 constexpr uint32_t kQosMaxAlpha = 32;
 constexpr uint32_t kQosUnsplit = 0xFFFFu; // block field of a queue entry that runs unsplit (f4)
 struct QosArgs {
@@ -152,8 +153,8 @@ struct QosArgs {
     const uint32_t* uns;           // [n_types] unsplit latency T per type (policy 2 only)
     const uint32_t* ref;           // [n_types] latency reference of violations / RR (= ext unless the caller sets it)
 };
-size_t qos_smem_bytes(const QosArgs& a);
-cudaError_t launch_qos(const QosArgs& a, cudaStream_t st);
+size_t qos_smem_bytes(const QosArgs& a, uint32_t qcap);
+cudaError_t launch_qos(const QosArgs& a, cudaStream_t st, uint32_t qcap);
 
 cudaError_t launch_exh_table(const ExhArgs& a, cudaStream_t st);
 cudaError_t launch_exh(const ExhArgs& a, int mode, uint32_t grid, cudaStream_t st);

@@ -21,7 +21,7 @@ namespace splitga {
 
 // kConverge: advance every replica of a warp by one event per loop trip and re-converge the warp
 // after it (policy 2; see the loop).  Policies 0/1 run the free-running loop, measured faster there.
-template <bool kConverge>
+template <bool kConverge, uint32_t QCAP>
 __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
 {
     extern __shared__ __align__(16) uint8_t smem[];
@@ -30,10 +30,10 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     uint32_t* s_alpha = s_ext + a.n_types;                // [n_alpha]
     uint32_t* s_blk = s_alpha + a.n_alpha;                // [total blocks]
     const uint32_t nb = a.n_blocks_total;
-    uint32_t* q_req = s_blk + nb;                         // [kQosQueue][kQosThreads]
-    uint32_t* q_left = q_req + kQosQueue * kQosThreads;   // Ext_left (ns)
-    uint32_t* q_tb = q_left + kQosQueue * kQosThreads;    // type | next block << 16
-    uint32_t* s_viol = q_tb + kQosQueue * kQosThreads;    // [n_alpha][kQosThreads]
+    uint32_t* q_req = s_blk + nb;                         // [QCAP][kQosThreads]
+    uint32_t* q_left = q_req + QCAP * kQosThreads;        // Ext_left (ns)
+    uint32_t* q_tb = q_left + QCAP * kQosThreads;         // type | next block << 16
+    uint32_t* s_viol = q_tb + QCAP * kQosThreads;         // [n_alpha][kQosThreads]
     uint32_t* s_uns = s_viol + a.n_alpha * kQosThreads;   // [M] unsplit T (policy 2)
     uint32_t* s_ref = s_uns + a.n_types;                  // [M] latency reference of the statistics
     for (uint32_t j = threadIdx.x; j <= a.n_types; j += blockDim.x) s_off[j] = a.blk_off[j];
@@ -129,7 +129,7 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
                         left0 = off ? s_uns[m] : e;
                         tb0 = off ? (m | (kQosUnsplit << 16)) : m;
                     }
-                    if (n == kQosQueue) { err = 2u; break; }
+                    if (n == QCAP) { err = 2u; break; }
                     for (uint32_t j = n; j > pos; --j) {
                         Q(q_req, j) = Q(q_req, j - 1);
                         Q(q_left, j) = Q(q_left, j - 1);
@@ -174,17 +174,20 @@ __global__ void __launch_bounds__(kQosThreads) qos_kernel(QosArgs a)
     a.rr[2 * r + 1] = rq;
 }
 
-size_t qos_smem_bytes(const QosArgs& a)
+size_t qos_smem_bytes(const QosArgs& a, uint32_t qcap)
 {
-    return 4 * ((size_t)2 * a.n_types + 1 + a.n_alpha + a.n_blocks_total) + 4 * (size_t)3 * kQosQueue * kQosThreads +
+    return 4 * ((size_t)2 * a.n_types + 1 + a.n_alpha + a.n_blocks_total) + 4 * (size_t)3 * qcap * kQosThreads +
            4 * (size_t)a.n_alpha * kQosThreads + 8 * (size_t)a.n_types + 16;
 }
 
-cudaError_t launch_qos(const QosArgs& a, cudaStream_t st)
+// qcap: kQosQueue (the fast form: many CTAs per SM) or kQosQueueBig (the host's re-run after an overflow)
+cudaError_t launch_qos(const QosArgs& a, cudaStream_t st, uint32_t qcap)
 {
     if (a.n_rep == 0) return cudaSuccess;
-    const size_t sm = qos_smem_bytes(a);
-    const auto kern = (a.policy == 2u) ? qos_kernel<true> : qos_kernel<false>;
+    const size_t sm = qos_smem_bytes(a, qcap);
+    const bool big = qcap > kQosQueue;
+    const auto kern = (a.policy == 2u) ? (big ? qos_kernel<true, kQosQueueBig> : qos_kernel<true, kQosQueue>)
+                                       : (big ? qos_kernel<false, kQosQueueBig> : qos_kernel<false, kQosQueue>);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
     const uint32_t grid = (uint32_t)((a.n_rep + kQosThreads - 1) / kQosThreads);

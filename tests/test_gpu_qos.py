@@ -96,11 +96,13 @@ def test_error_paths(S):
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate(blocks, a, t, [2000], 1)
     assert e.value.code == S.SPLIT_E_RANGE
-    a = torch.zeros((40, 1), dtype=torch.int64, device="cuda")            # 40 simultaneous: > 32 pending
-    t = torch.zeros((40, 1), dtype=torch.int32, device="cuda")
+    a = torch.zeros((200, 1), dtype=torch.int64, device="cuda")           # 200 simultaneous: > 160 pending
+    t = torch.zeros((200, 1), dtype=torch.int32, device="cuda")
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate(blocks, a, t, [2000], 0)
     assert e.value.code == S.SPLIT_E_RANGE
+    a = torch.zeros((40, 1), dtype=torch.int64, device="cuda")
+    t = torch.zeros((40, 1), dtype=torch.int32, device="cuda")
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate([[0]], a, t, [2000], 0)                        # zero-length block
     assert e.value.code == S.SPLIT_E_RANGE
@@ -192,3 +194,26 @@ def test_elastic_error_paths(S):
     with pytest.raises(S.SplitError) as e:
         S.split_qos_simulate([[5]], a, t, [2000], 3)                                   # no such policy
     assert e.value.code == S.SPLIT_E_INVAL
+
+
+@pytest.mark.parametrize("pol", [Q.FIFO, Q.ALG1, Q.ELASTIC])
+def test_overloaded_queue_rerun(S, pol):
+    """More than 32 pending requests in some replicas (bursts of simultaneous arrivals, a load
+    Table 2 never reaches): the library re-runs the batch with the 160-entry queue; every replica
+    still matches the literal oracle (round 1 returned SPLIT_E_RANGE here)."""
+    blocks = wl.random_blocks(3, seed=11, k_hi=4, lo=1_000_000, hi=5_000_000)
+    rng = np.random.default_rng(11)
+    n_rep, n_req = 8, 120
+    arr = np.sort(rng.integers(0, 40_000_000, size=(n_rep, n_req)), axis=1).astype(np.int64)
+    arr[:, :60] = 1000                                    # a burst of 60 simultaneous arrivals
+    arr = np.sort(arr, axis=1)
+    ty = rng.integers(0, 3, size=(n_rep, n_req)).astype(np.int32)
+    uns = [max(1, sum(b) - 50_000) for b in blocks]
+    kw = dict(unsplit=uns, d_max=40, s_max=30) if pol == Q.ELASTIC else {}
+    te, viol, rr = S.split_qos_simulate(blocks, torch.from_numpy(np.ascontiguousarray(arr.T)).cuda(),
+                                        torch.from_numpy(np.ascontiguousarray(ty.T)).cuda(), ALPHAS, pol, **kw)
+    torch.cuda.synchronize()
+    te = np.ascontiguousarray(te.cpu().numpy().T)
+    for r in range(n_rep):
+        args = (uns, 40, 30) if pol == Q.ELASTIC else ()
+        assert [int(x) for x in te[r]] == Q.simulate(blocks, arr[r].tolist(), ty[r].tolist(), pol, *args)
