@@ -364,6 +364,116 @@ __global__ void __launch_bounds__(NW_ * 32, NW_ == 8 ? 5 : (48 / NW_ > 0 ? 48 / 
 }
 
 // ------------------------------------------------------------------------
+// K1, grouped form (W = 16): one CTA holds NG independent groups of NWG warps.
+// Each group is what one CTA of eval_batch_w_kernel<16, NWG, 1, 1, 0, true>
+// is -- its own swizzled chunk buffer, mbarrier, histogram and sorted order,
+// synchronised by its own named barrier (bar.sync 1 + g) -- but the groups
+// share one staged chain table, so an SM holds more warps and more
+// independent barrier domains in the same shared memory.
+// ------------------------------------------------------------------------
+template <int NWG, int NG>
+struct GrpCfg {
+    static constexpr uint32_t CHUNK = NWG * 32, H = 32;
+    static constexpr uint32_t kBoxes = (CHUNK + 255u) / 256u, kBoxRows = CHUNK / kBoxes;
+    static size_t smem(uint32_t po_bytes)
+    {
+        return (size_t)NG * CHUNK * 128 + po_bytes + 8 * (1 + NG + 1) + (size_t)NG * (CHUNK * 6 + 128) + 64;
+    }
+};
+
+__device__ __forceinline__ void named_bar(uint32_t id, uint32_t nthreads)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+template <int NWG, int NG>
+__global__ void __launch_bounds__(NWG * NG * 32, (48 / (NWG * NG)) > 0 ? 48 / (NWG * NG) : 1)
+    eval_grp_kernel(ChainDev ch, const uint64_t* __restrict__ bits, uint64_t n_cand, double* __restrict__ out,
+                    const __grid_constant__ CUtensorMap tmap)
+{
+    using Cfg = GrpCfg<NWG, NG>;
+    constexpr uint32_t CHUNK = Cfg::CHUNK, H = Cfg::H, NTG = NWG * 32;
+    static_assert(CHUNK % 8 == 0 && Cfg::kBoxRows * Cfg::kBoxes == CHUNK, "swizzled chunk geometry");
+    extern __shared__ __align__(1024) uint8_t smem_grp[];
+    const uint32_t tid = threadIdx.x, g = tid / NTG, gt = tid % NTG, lane = tid & 31u, gwarp = gt >> 5;
+    uint32_t* buf = (uint32_t*)smem_grp + (size_t)g * CHUNK * H;          // this group's chunk buffer
+    const uint2* spo = (const uint2*)(smem_grp + (size_t)NG * CHUNK * 128);
+    uint64_t* mbar = (uint64_t*)((const uint8_t*)spo + ch.po_bytes);       // [0] chain, [1 + g] groups
+    uint8_t* gbase = (uint8_t*)(mbar + 1 + NG + 1) + (size_t)g * (CHUNK * 6 + 128);
+    uint32_t* s_occ = (uint32_t*)gbase;                                    // [CHUNK]
+    uint32_t* s_hist = s_occ + CHUNK;                                      // [32]
+    uint16_t* s_perm = (uint16_t*)(s_hist + 32);                           // [CHUNK]
+    if (tid == 0)
+        for (uint32_t q = 0; q < NG; ++q) mbar_init(mbar + 1 + q, 1);
+    if (gt < 32) s_hist[gt] = 0;
+    stage_bulk((void*)spo, ch.po, ch.po_bytes, mbar);                      // includes a __syncthreads
+    const uint32_t npos = ch.n - 1, qfull = npos >> 5;
+    const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
+    const uint32_t validocc = (qfull >= 32u) ? ~0u : ((1u << qfull) - 1u);
+    const uint32_t spo_s = opaque32(smem_u32(spo));
+    const uint64_t n_chunks = (n_cand + CHUNK - 1) / CHUNK;
+    const uint64_t stride = (uint64_t)gridDim.x * NG;
+    uint64_t c = (uint64_t)blockIdx.x * NG + g;
+    auto issue = [&](uint64_t cc) {
+        if (gt == 0 && cc < n_chunks) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_expect_tx(mbar + 1 + g, CHUNK * 128u);
+#pragma unroll
+            for (uint32_t x = 0; x < Cfg::kBoxes; ++x) {
+                const int32_t y = (int32_t)(cc * CHUNK + x * Cfg::kBoxRows);
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                    ::"r"(smem_u32(buf + x * Cfg::kBoxRows * H)), "l"(&tmap), "r"(0), "r"(y), "r"(smem_u32(mbar + 1 + g))
+                    : "memory");
+            }
+        }
+    };
+    issue(c);
+    uint32_t ph = 0;
+    for (; c < n_chunks; c += stride) {
+        const uint64_t row0 = c * CHUNK;
+        const uint32_t rows = (uint32_t)((n_cand - row0) < CHUNK ? (n_cand - row0) : CHUNK);
+        mbar_wait(mbar + 1 + g, ph);
+        ph ^= 1u;
+        uint32_t key = 0, flags = 0x4000u;
+        if (gt < rows) {
+            uint32_t cuts;
+            const uint32_t occ = row_occupancy<16, false, true>(buf + gt * H, lane, validocc, qfull, lastm, cuts);
+            s_occ[gt] = occ;
+            const uint32_t ne = __popc(occ);
+            flags = (ne < ch.k_max && cuts < ch.k_max) ? 0u : 0x8000u;
+            key = flags ? 0u : min(cuts, 31u);
+        }
+        const uint32_t rank = atomicAdd(&s_hist[key], 1u);
+        named_bar(1 + g, NTG);
+        {
+            const uint32_t hv = s_hist[lane];
+            uint32_t inc = hv;
+#pragma unroll
+            for (uint32_t o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, inc, o);
+                if (lane >= o) inc += y;
+            }
+            const uint32_t start = __shfl_sync(0xFFFFFFFFu, inc - hv, key);
+            s_perm[start + rank] = (uint16_t)(gt | flags);
+        }
+        named_bar(1 + g, NTG);
+        if (gt < 32) s_hist[gt] = 0;
+        {
+            const uint32_t pe = s_perm[32u * gwarp + lane];
+            const uint32_t r = pe & 0x3FFFu;
+            if (!(pe & 0x4000u)) {
+                const double f = (pe & 0x8000u) ? -CUDART_INF
+                                                : walk_row<true>(ch, s_occ[r], smem_u32(buf + r * H), r, spo_s);
+                __stcs(out + row0 + r, f);
+            }
+        }
+        named_bar(1 + g, NTG);                    // this group's buffer, occupancy masks and order released
+        issue(c + stride);
+    }
+}
+
+// ------------------------------------------------------------------------
 // Small kernels
 // ------------------------------------------------------------------------
 __global__ void eval_stats_kernel(ChainDev ch, const uint64_t* bits, int64_t* st_out, double* f_out)
@@ -404,7 +514,18 @@ __global__ void selftest_dexp_kernel(const double* in, uint32_t n, double* out)
 struct EvalVariant {
     void* fn;
     uint32_t W, NW, RPT, NB, SWZ;
+    uint32_t NG = 0;                                  // grouped kernel: NG groups of NW warps per CTA
+    size_t (*grp_smem)(uint32_t) = nullptr;
 };
+
+template <int NWG, int NG>
+static EvalVariant eval_grp_variant()
+{
+    EvalVariant v{(void*)eval_grp_kernel<NWG, NG>, 16u, (uint32_t)NWG, 1u, 1u, 1u};
+    v.NG = NG;
+    v.grp_smem = &GrpCfg<NWG, NG>::smem;
+    return v;
+}
 
 template <int W, int NW, int RPT, int NB, int KEY = 0, bool SWZ = false>
 static EvalVariant eval_variant()
@@ -455,7 +576,7 @@ static bool make_row_tmap(CUtensorMap* m, const uint64_t* bits, uint64_t n_cand,
 template <int W>
 static EvalVariant eval_default()
 {
-    if constexpr (W == 16) return eval_variant<W, 11, 1, 1, 0, true>();   // 4 CTAs x 11 warps per SM
+    if constexpr (W == 16) return eval_grp_variant<6, 4>();   // 2 CTAs x 4 groups x 6 warps per SM
     else if constexpr (W >= 12) return eval_variant<W, 15, 1, 1>();
     else if constexpr (W >= 6) return eval_variant<W, 8, 2, 1>();
     else return eval_variant<W, 8, 2, 2>();
@@ -470,10 +591,22 @@ static EvalVariant eval_pick(uint32_t W)
     if (W == 16 && sel >= 0) {
         switch (sel) {
         case 100: return eval_variant<16, 15, 1, 1>();            // the round-1 default (bulk copies, no swizzle)
+        case 120: return eval_variant<16, 11, 1, 1, 0, true>();   // one group per CTA, 4 CTAs x 11 warps
         case 101: return eval_variant<16, 15, 1, 1, 1, true>();
         case 102: return eval_variant<16, 16, 1, 1, 0, true>();
         case 103: return eval_variant<16, 12, 1, 1, 0, true>();
         case 104: return eval_variant<16, 8, 2, 1, 0, true>();
+        case 400: return eval_grp_variant<6, 4>();     // 2 CTAs x 4 groups x 6 warps per SM
+        case 401: return eval_grp_variant<5, 4>();
+        case 402: return eval_grp_variant<8, 3>();
+        case 403: return eval_grp_variant<11, 2>();
+        case 404: return eval_grp_variant<4, 6>();
+        case 405: return eval_grp_variant<12, 2>();
+        case 406: return eval_grp_variant<8, 2>();
+        case 410: return eval_grp_variant<5, 5>();
+        case 411: return eval_grp_variant<7, 3>();
+        case 412: return eval_grp_variant<3, 8>();
+        case 413: return eval_grp_variant<6, 3>();
         case 110: return eval_variant<16, 10, 1, 1, 0, true>();
         case 111: return eval_variant<16, 11, 1, 1, 0, true>();
         case 113: return eval_variant<16, 13, 1, 1, 0, true>();
@@ -526,11 +659,12 @@ cudaError_t launch_eval_batch(const ChainDev& ch, const uint64_t* bits, uint64_t
         if (n_cand >= (1ull << 31) || !make_row_tmap(&tmap, bits, n_cand, chunk / nbox))
             v = eval_variant<16, 15, 1, 1>();
     }
-    const size_t sm = v.RPT ? eval_smem_of(ch, v)
-                            : (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
+    const size_t sm = v.NG ? v.grp_smem(ch.po_bytes)
+                           : v.RPT ? eval_smem_of(ch, v)
+                                   : (size_t)(ch.p_words + ch.o_words) * 4 + 16 + (size_t)kEvalWarps * 32 * (ch.W | 1u) * 8;
     cudaError_t e = cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    const uint32_t nt = 32u * v.NW;
+    const uint32_t nt = 32u * v.NW * (v.NG ? v.NG : 1u);
     int per_sm = 0;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v.fn, (int)nt, sm);
     if (e != cudaSuccess) return e;
