@@ -26,8 +26,7 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
-# stdout carries exactly one JSON line: NCCL's own messages (e.g. its version banner) go to stderr
-os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+
 
 import numpy as np  # noqa: E402
 
@@ -274,6 +273,15 @@ def run_reference(args):
     return 0
 
 
+def _json_stdout():
+    """stdout carries exactly one JSON line: keep a handle on the real stdout for it and point file
+    descriptor 1 at stderr, so native libraries (NCCL's version banner, ...) cannot add lines."""
+    sys.stdout.flush()
+    real = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
+    return real
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -294,6 +302,7 @@ def main():
         args.warmup = 3
     if args.impl == "reference":
         return run_reference(args)
+    json_out = _json_stdout()
 
     import torch
     import torch.distributed as dist
@@ -440,19 +449,24 @@ def main():
         for _ in range(3):
             h5.eval_batch(bits, C5_EVAL_N, fout)
         torch.cuda.synchronize()
-        e0 = [torch.cuda.Event(enable_timing=True) for _ in range(10)]
-        e1 = [torch.cuda.Event(enable_timing=True) for _ in range(10)]
-        for i in range(10):
-            flush.fill_(i)
-            e0[i].record(stream)
-            h5.eval_batch(bits, C5_EVAL_N, fout)
-            e1[i].record(stream)
-        torch.cuda.synchronize()
-        ms = [a.elapsed_time(b) for a, b in zip(e0, e1)]
-        ms_avg = sum(ms) / len(ms)
+        # the 2.3 GB of C5 rows are far larger than L2, so consecutive launches need no flush between
+        # them: 20 launches back to back between two events on the launching stream (launch-to-launch gaps
+        # included), a few times, the median
+        reps_ms = []
+        for _ in range(5):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(20):
+                h5.eval_batch(bits, C5_EVAL_N, fout)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            reps_ms.append(e0.elapsed_time(e1) / 20)
+        ms_avg = statistics.median(reps_ms)
         bpc = eval_bytes_per_candidate(W5)
         gbs = bpc * C5_EVAL_N / (ms_avg / 1000.0) / 1e9
-        out["eval_roofline"] = {"kernel": "eval_batch_w_kernel (K1, split_eval_batch)", "bound": "hbm",
+        out["eval_roofline"] = {"kernel": "eval_grp_kernel<6, 4> (K1, split_eval_batch at W = 16)", "bound": "hbm",
+                                "timing": "median of 5 x 20 back-to-back launches on the launching stream; inputs "
+                                          "(2.3 GB) larger than L2, no flush",
                                 "frac": gbs / peaks["hbm_gbs"], "achieved": gbs, "peak": peaks["hbm_gbs"],
                                 "unit": "GB/s", "traffic": _profile_traffic("eval_batch_kernel_c5"),
                                 "algorithmic": f"{eval_bytes_per_candidate(W5)} B/candidate x 2^24",
@@ -460,7 +474,7 @@ def main():
         out["eval_batch"] = {
             "workload": "C5: synthetic 1024-op chain (W=16), N=2^24 candidates, k ~ U[2,32]",
             "evals_per_s": C5_EVAL_N / (ms_avg / 1000.0), "ms_per_launch": ms_avg,
-            "roofline": {"bound": "hbm", "kernel": "eval_batch_kernel", "achieved": gbs, "peak": peaks["hbm_gbs"],
+            "roofline": {"bound": "hbm", "kernel": "eval_grp_kernel", "achieved": gbs, "peak": peaks["hbm_gbs"],
                          "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"], "peak_src": peaks["src"],
                          "traffic": _profile_traffic("eval_batch_kernel_c5"),
                          "algorithmic_bytes_per_candidate": bpc}}
@@ -694,7 +708,7 @@ def main():
     if comm:
         S.split_comm_destroy(comm)
     if rank == 0:
-        print(json.dumps(out), flush=True)
+        print(json.dumps(out), file=json_out, flush=True)
     if world > 1:
         dist.destroy_process_group()
     return 0

@@ -12,7 +12,7 @@ timeout 900 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_ful
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-ga-big --no-qos --no-c3 --no-c4 > gpurun_out/launch_bench.log 2>&1
 N=/tmp/ncu
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:ga_kernel -s 1 -c 1 -o $N/prof_ga -f python tools/prof_driver.py ga 2 500 > gpurun_out/ncu_ga.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval_batch -s 1 -c 1 -o $N/prof_eval -f python tools/prof_driver.py eval 2 > gpurun_out/ncu_eval.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval_ -s 1 -c 1 -o $N/prof_eval -f python tools/prof_driver.py eval 2 > gpurun_out/ncu_eval.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:ga_kernel -s 1 -c 1 -o $N/prof_ga_1m -f python tools/prof_driver.py ga_1m 1 20 > gpurun_out/ncu_ga_1m.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:ga_kernel -s 1 -c 1 -o $N/prof_ga_4m -f python tools/prof_driver.py ga_big 1 20 > gpurun_out/ncu_ga_4m.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:qos_kernel -s 1 -c 1 -o $N/prof_qos -f python tools/prof_driver.py qos 2 > gpurun_out/ncu_qos.log 2>&1
