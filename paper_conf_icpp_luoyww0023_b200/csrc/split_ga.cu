@@ -108,49 +108,49 @@ __device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch
 // the trip count is the child's cut count rather than a per-word maximum.
 // Same integer statistics and Eq. 2 tail as eval_walk (R3, R5').
 template <int WT>
-__device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
-                                                   const Row<WT>& r)
+__device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, uint32_t spo_s, const Row<WT>& r, uint32_t cuts)
 {
     constexpr int NH = 2 * WT;
     uint32_t h[NH];
-    uint32_t occ = 0, cuts = 0;
+    uint32_t occ = 0;
 #pragma unroll
     for (int i = 0; i < NH; ++i) {
         const uint64_t wv = (i / 2 < (int)ch.W) ? (r.w[i / 2] & word_mask(ch, i / 2)) : 0ull;
         h[i] = (uint32_t)(wv >> (32 * (i & 1)));
         occ |= (h[i] != 0u ? 1u : 0u) << i;
-        cuts += __popc(h[i]);
     }
     const uint32_t k = cuts + 1;
     if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
-    uint32_t endP = ch.T, OV = 0, v = 0, qb = 0;
+    uint32_t endP = ch.T, OV = 0, v = 0, tb = spo_s;
     uint64_t S2 = 0;
     for (uint32_t j = 0; j < cuts; ++j) {
-        if (v == 0u) {
-            const uint32_t q = bfind32(occ);
-            occ ^= 1u << q;
-            // select tree over the halves by the bits of q
-            uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
+        // refill (predicated): the next non-empty half when v is exhausted, chosen by a
+        // select tree over the bits of q (never a runtime register index)
+        const uint32_t q = bfind32(occ);
+        const bool need = (v == 0u);
+        uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
 #pragma unroll
-            for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
-            if constexpr (NH == 2) v = t1[0];
-            else if constexpr (NH == 4) v = (q & 2u) ? t1[1] : t1[0];
-            else {
-                const uint32_t a0 = (q & 2u) ? t1[1] : t1[0];
-                const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
-                v = (q & 4u) ? a1 : a0;
-            }
-            qb = q << 5;
+        for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
+        uint32_t hv;
+        if constexpr (NH == 2) hv = t1[0];
+        else if constexpr (NH == 4) hv = (q & 2u) ? t1[1] : t1[0];
+        else {
+            const uint32_t a0 = (q & 2u) ? t1[1] : t1[0];
+            const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
+            hv = (q & 4u) ? a1 : a0;
         }
+        v = need ? hv : v;
+        occ = need ? (occ & bmsk32(q)) : occ;
+        tb = need ? spo_s + (q << 8) : tb;
         const uint32_t bt = bfind32(v);
-        v ^= 1u << bt;
-        const uint32_t p = qb + bt;
-        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
-        const uint32_t Pp = sP[p + 1], op = sO[p];
-        const uint32_t t = endP - Pp + op;
+        v &= bmsk32(bt);
+        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3):
+        // one LDS.64 of the staged pair {P[p+1], ovh[p]}
+        const uint2 e = lds64(tb + 8u * bt);
+        const uint32_t t = endP - e.x + e.y;
         S2 += (uint64_t)t * t;
-        OV += op;
-        endP = Pp;
+        OV += e.y;
+        endP = e.x;
     }
     S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
     const uint64_t S1 = (uint64_t)ch.T + OV;
@@ -160,14 +160,14 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uin
 
 // Wide rows (4 < W <= 16): the row's 32-bit halves go to this thread's slot of
 // shared memory (odd pitch 2W+1: conflict-free), then one loop iteration per
-// cut, descending, refilling from the occupancy mask -- the trip count is the
-// child's cut count, not a per-word maximum over the warp's lanes.  Same
-// integer statistics and Eq. 2 tail as eval_walk (R3, R5').
+// cut, descending, with a predicated refill from the occupancy mask -- the trip
+// count is the child's cut count, not a per-word maximum over the warp's
+// lanes.  Same integer statistics and Eq. 2 tail as eval_walk (R3, R5').
 template <int WT>
-__device__ __forceinline__ double eval_wide(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
-                                            const Row<WT>& r, uint32_t* my)
+__device__ __forceinline__ double eval_wide(const ChainDev& ch, uint32_t spo_s, const Row<WT>& r, uint32_t* my,
+                                            uint32_t cuts)
 {
-    uint32_t occ = 0, cuts = 0;
+    uint32_t occ = 0;
 #pragma unroll
     for (int i = 0; i < WT; ++i) {
         if (i < (int)ch.W) {
@@ -175,30 +175,28 @@ __device__ __forceinline__ double eval_wide(const ChainDev& ch, const uint32_t* 
             const uint32_t lo = (uint32_t)wv, hi = (uint32_t)(wv >> 32);
             my[2 * i] = lo;
             my[2 * i + 1] = hi;
-            occ |= ((lo != 0u ? 1u : 0u) | (hi != 0u ? 2u : 0u)) << (2 * i);
-            cuts += __popc(lo) + __popc(hi);
+            occ |= (min(lo, 1u) | (min(hi, 1u) << 1)) << (2 * i);
         }
     }
     const uint32_t k = cuts + 1;
     if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
-    uint32_t endP = ch.T, OV = 0, v = 0, qb = 0;
+    const uint32_t my_s = smem_u32(my);
+    uint32_t endP = ch.T, OV = 0, v = 0, tb = spo_s;
     uint64_t S2 = 0;
     for (uint32_t j = 0; j < cuts; ++j) {
-        if (v == 0u) {
-            const uint32_t q = bfind32(occ);
-            occ ^= 1u << q;
-            v = my[q];
-            qb = q << 5;
-        }
+        const uint32_t q = bfind32(occ);
+        const bool need = (v == 0u);
+        occ = need ? (occ & bmsk32(q)) : occ;
+        v = lds32_if(need, my_s + 4u * q, v);
+        tb = need ? spo_s + (q << 8) : tb;
         const uint32_t bt = bfind32(v);
-        v ^= 1u << bt;
-        const uint32_t p = qb + bt;
+        v &= bmsk32(bt);
         // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
-        const uint32_t Pp = sP[p + 1], op = sO[p];
-        const uint32_t t = endP - Pp + op;
+        const uint2 e = lds64(tb + 8u * bt);
+        const uint32_t t = endP - e.x + e.y;
         S2 += (uint64_t)t * t;
-        OV += op;
-        endP = Pp;
+        OV += e.y;
+        endP = e.x;
     }
     S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
     const uint64_t S1 = (uint64_t)ch.T + OV;
@@ -206,14 +204,25 @@ __device__ __forceinline__ double eval_wide(const ChainDev& ch, const uint32_t* 
     return eq2(k, V, OV, ch);
 }
 
+// spo_s: shared address of the staged {P[p+1], ovh[p]} pairs; cuts_known: the row's
+// cut count when the caller has it (else ~0u)
 template <int WT>
 __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
-                                            const Row<WT>& r, Stats* st, uint32_t* srow = nullptr)
+                                            const Row<WT>& r, Stats* st, uint32_t* srow = nullptr,
+                                            uint32_t spo_s = 0u, uint32_t cuts_known = ~0u)
 {
-    if constexpr (WT <= 4) {
-        if (!st) return eval_regs_narrow<WT>(ch, sP, sO, r);
-    } else if constexpr (WT <= 16) {
-        if (!st && srow) return eval_wide<WT>(ch, sP, sO, r, srow);
+    if constexpr (WT <= 16) {
+        if (!st && spo_s && (WT <= 4 || srow)) {
+            uint32_t c = cuts_known;
+            if (c == ~0u) {
+                c = 0;
+#pragma unroll
+                for (int w = 0; w < WT; ++w)
+                    if (w < (int)ch.W) c += __popcll(r.w[w] & word_mask(ch, w));
+            }
+            if constexpr (WT <= 4) return eval_regs_narrow<WT>(ch, spo_s, r, c);
+            else return eval_wide<WT>(ch, spo_s, r, srow, c);
+        }
     }
     // same arithmetic as eval_walk, with the word loop unrolled over the register row
     uint32_t cuts = 0;
@@ -458,7 +467,8 @@ struct RecCache {
 
 struct Smem {
     uint32_t* chain;
-    uint64_t* mbar;       // [0]: chain staging, [1]: leader loads (reused every generation)
+    uint64_t* mbar;       // [0]: chain staging, [1]: leader loads (reused every generation), [2]: pair table
+    uint2* po;            // staged {P[p+1], ovh[p]} pairs (one LDS.64 per cut in the fused eval)
     uint32_t* hist;       // [I][256]
     SelState* sel;        // [I]
     BestRef* scratch;     // 33 BestRow<WT>
@@ -488,7 +498,8 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     auto take = [&](size_t bytes) { size_t o = off; off = align16(off + bytes); return base + o; };
     uint8_t* p;
     p = take((size_t)(a.ch.p_words + a.ch.o_words) * 4); if (s) s->chain = (uint32_t*)p;
-    p = take(16); if (s) s->mbar = (uint64_t*)p;
+    p = take(32); if (s) s->mbar = (uint64_t*)p;
+    p = take(a.ch.po_bytes); if (s) s->po = (uint2*)p;
     p = take((size_t)a.I * 256 * 4); if (s) s->hist = (uint32_t*)p;
     p = take((size_t)a.I * sizeof(SelState)); if (s) s->sel = (SelState*)p;
     p = take(33 * (16 + 8 * (size_t)wt_of(a.ch.W))); if (s) s->scratch = (BestRef*)p;
@@ -753,6 +764,211 @@ __device__ void cta_select_sorted(const uint64_t* key, const uint32_t* idx, uint
         ox[r] = xj;
     }
     __syncthreads();
+}
+
+// ------------------------------------------------------------------------
+// Small selections (sync points): sorts instead of the radix select, which
+// pays ~1.2 us per 8-bit digit and needs up to 12 digits when the keys of a
+// converged island tie.  Branch-free compares (the branchy form serialises on
+// every shuffle).  Sentinel entries (key 0, idx ~0) sort last: no fitness key
+// is 0.
+// ------------------------------------------------------------------------
+__device__ __forceinline__ bool gt_nb(uint64_t ka, uint32_t ia, uint64_t kb, uint32_t ib)
+{
+    return (ka > kb) | ((ka == kb) & (ia < ib));
+}
+
+// one warp: bitonic sort of 32*PER entries in registers (entry lane*PER + e) into the
+// ranking order of comp_gt; strides below PER inside a lane, the others by shuffles
+template <int PER>
+__device__ __forceinline__ void warp_bitonic_desc(uint64_t (&k)[PER], uint32_t (&x)[PER], uint32_t lane)
+{
+    constexpr uint32_t NE = 32u * PER;
+#pragma unroll
+    for (uint32_t size = 2; size <= NE; size <<= 1) {
+#pragma unroll
+        for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+            if (stride >= (uint32_t)PER) {                                // across lanes
+                const uint32_t pl = stride / PER;
+                const bool lower = (lane & pl) == 0u;
+                uint64_t ko[PER];
+                uint32_t xo[PER];
+#pragma unroll
+                for (int e = 0; e < PER; ++e) {
+                    ko[e] = __shfl_xor_sync(0xFFFFFFFFu, k[e], pl);
+                    xo[e] = __shfl_xor_sync(0xFFFFFFFFu, x[e], pl);
+                }
+#pragma unroll
+                for (int e = 0; e < PER; ++e) {
+                    const bool desc = ((lane * PER + e) & size) == 0u;
+                    // the lower position of a pair keeps the greater entry when descending (one
+                    // compare, flipped by xor: a branch here diverges and serialises the warp; equal
+                    // entries are identical sentinels, so swapping them is harmless)
+                    const bool take = gt_nb(ko[e], xo[e], k[e], x[e]) != (lower != desc);
+                    k[e] = take ? ko[e] : k[e];
+                    x[e] = take ? xo[e] : x[e];
+                }
+            } else {                                                      // inside a lane
+#pragma unroll
+                for (int e = 0; e < PER; ++e) {
+                    if ((e & stride) != 0u) continue;
+                    const int f = e | (int)stride;
+                    const bool desc = ((lane * PER + e) & size) == 0u;
+                    const bool sw = gt_nb(k[f], x[f], k[e], x[e]) == desc;
+                    const uint64_t ke = k[e], kf = k[f];
+                    const uint32_t xe = x[e], xf = x[f];
+                    k[e] = sw ? kf : ke; k[f] = sw ? ke : kf;
+                    x[e] = sw ? xf : xe; x[f] = sw ? xe : xf;
+                }
+            }
+        }
+    }
+}
+
+// one warp: sort entries [0, n) of key/idx (n <= 32*PER); the first m in ranking order to ok/ox
+template <int PER>
+__device__ __forceinline__ void warp_sort_write(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t m,
+                                                uint64_t* ok, uint32_t* ox, uint32_t lane)
+{
+    uint64_t k[PER];
+    uint32_t x[PER];
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+        const uint32_t j = lane * PER + e;
+        k[e] = j < n ? key[j] : 0ull;
+        x[e] = j < n ? idx[j] : ~0u;
+    }
+    warp_bitonic_desc<PER>(k, x, lane);
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+        const uint32_t j = lane * PER + e;
+        if (j < m) { ok[j] = k[e]; ox[j] = x[e]; }
+    }
+}
+
+// one warp: the m largest (ranking order) of the union of the lanes' lists -- each lane
+// holds PER entries sorted in ranking order -- by m rounds of a butterfly argmax over the
+// lanes' heads; the lane whose head won pops it.  The r-th result goes to ok/ox[r].
+template <int PER>
+__device__ __forceinline__ void warp_topm_lists(uint64_t (&k)[PER], uint32_t (&x)[PER], uint32_t m, uint64_t* ok,
+                                                uint32_t* ox, uint32_t lane)
+{
+    for (uint32_t r = 0; r < m; ++r) {
+        uint64_t bk = k[0];
+        uint32_t bx = x[0];
+#pragma unroll
+        for (uint32_t off = 16; off > 0; off >>= 1) {
+            const uint64_t ko = __shfl_xor_sync(0xFFFFFFFFu, bk, off);
+            const uint32_t xo = __shfl_xor_sync(0xFFFFFFFFu, bx, off);
+            const bool take = gt_nb(ko, xo, bk, bx);
+            bk = take ? ko : bk;
+            bx = take ? xo : bx;
+        }
+        if (lane == 0) { ok[r] = bk; ox[r] = bx; }
+        const bool pop = (k[0] == bk) & (x[0] == bx);    // composites are distinct (sentinels never win)
+#pragma unroll
+        for (int e = 0; e + 1 < PER; ++e) { k[e] = pop ? k[e + 1] : k[e]; x[e] = pop ? x[e + 1] : x[e]; }
+        k[PER - 1] = pop ? 0ull : k[PER - 1];
+        x[PER - 1] = pop ? ~0u : x[PER - 1];
+    }
+}
+
+// All 512 threads: the m largest (m <= 8) of 2048 entries in ranking order: every warp takes the top 8 of its
+// 128 (lane-local sort of 4, then warp_topm_lists), one warp the top m of the 16 x 8.
+// tk/tx: 128-entry scratch.  The result goes to ok/ox[0..m).
+__device__ __forceinline__ void cta_top8_of_2048(const uint64_t* key, const uint32_t* idx, uint32_t m, uint64_t* tk,
+                                                 uint32_t* tx, uint64_t* ok, uint32_t* ox)
+{
+    const uint32_t w = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+    {
+        uint64_t k[4];
+        uint32_t x[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) { k[e] = key[128u * w + 32u * e + lane]; x[e] = idx[128u * w + 32u * e + lane]; }
+        // sorting network of 4 inside the lane: (0,1)(2,3)(0,2)(1,3)(1,2)
+        auto cx = [&](int a, int b) {
+            const bool sw = gt_nb(k[b], x[b], k[a], x[a]);
+            const uint64_t ka = k[a], kb = k[b];
+            const uint32_t xa = x[a], xb = x[b];
+            k[a] = sw ? kb : ka; k[b] = sw ? ka : kb;
+            x[a] = sw ? xb : xa; x[b] = sw ? xa : xb;
+        };
+        cx(0, 1); cx(2, 3); cx(0, 2); cx(1, 3); cx(1, 2);
+        warp_topm_lists<4>(k, x, 8u, tk + 8u * w, tx + 8u * w, lane);
+    }
+    __syncthreads();
+    if (w == 0) {
+        uint64_t k[8];
+        uint32_t x[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            k[e] = lane < 16u ? tk[8u * lane + e] : 0ull;
+            x[e] = lane < 16u ? tx[8u * lane + e] : ~0u;
+        }
+        warp_topm_lists<8>(k, x, m, ok, ox, lane);
+    }
+    __syncthreads();
+}
+
+// All 512 threads: sort n <= 512 entries of key/idx (shared memory) in the ranking order
+// and write the first m to ok/ox.  One entry per thread: each warp sorts its 32 by a
+// register bitonic network, then four merge levels (runs of 32 -> 512) place every entry
+// at its own position plus its rank in the partner run (binary search; the left run wins
+// ties, so the sentinels never collide).  bk/bx: 512-entry scratch, distinct from ok/ox
+// (key/idx may be one of them).
+__device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t m, uint64_t* ok,
+                            uint32_t* ox, uint64_t* bk, uint32_t* bx)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    uint32_t t = threadIdx.x;
+    uint64_t k[1];
+    uint32_t x[1];
+    k[0] = t < n ? key[t] : 0ull;
+    x[0] = t < n ? idx[t] : ~0u;
+    warp_bitonic_desc<1>(k, x, lane);
+    __syncthreads();                             // key/idx may be overwritten below
+#pragma unroll
+    for (uint32_t L = 32; L < 512; L <<= 1) {
+        bk[t] = k[0];
+        bx[t] = x[0];
+        __syncthreads();
+        const uint32_t base = t & ~(2u * L - 1u), pos = t & (L - 1u);
+        const bool left = (t & L) == 0u;
+        const uint32_t ob = left ? base + L : base;
+        // left entries count the partner's strictly greater entries, right entries the
+        // greater-or-equal ones (a prefix of the partner run): branch-free binary lifting
+        uint32_t lo = 0;
+#pragma unroll
+        for (uint32_t step = L >> 1; step > 0; step >>= 1) {
+            const uint64_t km = bk[ob + lo + step - 1];
+            const uint32_t xm = bx[ob + lo + step - 1];
+            lo += (gt_nb(km, xm, k[0], x[0]) | (!left & !gt_nb(k[0], x[0], km, xm))) ? step : 0u;
+        }
+        {
+            const uint64_t km = bk[ob + lo];
+            const uint32_t xm = bx[ob + lo];
+            lo += (gt_nb(km, xm, k[0], x[0]) | (!left & !gt_nb(k[0], x[0], km, xm))) ? 1u : 0u;
+        }
+        __syncthreads();
+        t = base + pos + lo;
+    }
+    if (t < m) { ok[t] = k[0]; ox[t] = x[0]; }
+    __syncthreads();
+}
+
+// The k largest of n entries in ranking order to ok/ox[0..min(k, n)) -- the same result
+// as cta_select_sorted (composites are distinct): the merge sort above when n <= 512 and
+// the CTA has 512 threads, the radix select otherwise.  All threads of the CTA call it;
+// the inputs must be visible (a __syncthreads after they were written).  sm.okey/oidx
+// serve as scratch, as they do for the radix select.
+__device__ __noinline__ void select_sorted(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t k,
+                                           const Smem& sm, uint64_t* ok, uint32_t* ox)
+{
+    if (n > 512u || blockDim.x != 512u) {
+        cta_select_sorted(key, idx, n, k, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, ok, ox);
+        return;
+    }
+    cta_sort512(key, idx, n, min(k, n), ok, ox, sm.okey, sm.oidx);
 }
 
 // Leader CTA: sort the general-select output of island i in smem (ranking
@@ -1166,12 +1382,13 @@ __device__ __forceinline__ uint32_t tournament(const GaArgs& a, uint32_t gid, ui
     return best;
 }
 
+// returns the row's cut count after the repair
 template <int WT>
-__device__ __forceinline__ void repair(const GaArgs& a, Row<WT>& row, uint32_t gid, uint32_t g)
+__device__ __forceinline__ uint32_t repair(const GaArgs& a, Row<WT>& row, uint32_t gid, uint32_t g)
 {
     const ChainDev& ch = a.ch;
     uint32_t c = row_popc(row, ch);
-    if (c + 1 >= ch.k_min && c + 1 <= ch.k_max) return;
+    if (c + 1 >= ch.k_min && c + 1 <= ch.k_max) return c;
     Draws dr(gid, g, TAG_REPAIR, a.key0, a.key1);
     const uint32_t npos = ch.n - 1;
     if (c > ch.k_max - 1) {
@@ -1206,6 +1423,7 @@ __device__ __forceinline__ void repair(const GaArgs& a, Row<WT>& row, uint32_t g
         row_toggle_rank(row, ch, below(dr.next(), npos - a.front_skip - c), false, a.front_skip);
         ++c;
     }
+    return c;
 }
 
 template <int WT>
@@ -1265,7 +1483,7 @@ __device__ __forceinline__ ChildDraws child_draws(const GaArgs& a, uint32_t gid,
 template <int WT>
 __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint32_t g, uint32_t wl,
                                                const uint64_t* popc, const double* fitc, uint64_t* popn,
-                                               double* fitn, const uint32_t* sP, const uint32_t* sO,
+                                               double* fitn, const uint32_t* sP, const uint32_t* sO, uint32_t spo_s,
                                                const uint64_t* tau_ptr, uint32_t* s_ccnt, uint64_t* ckey,
                                                uint32_t* cidx, uint32_t* rcnt, uint32_t* ridx,
                                                const BestRow<WT>& snap, ChildDraws& pre, bool& have_pre,
@@ -1314,20 +1532,21 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         }
         if (tr) a.trace[(g - a.g_begin) * 16 + 9] = gtimer() + 0 * (A.w[0] ^ B.w[0]);
         if ((uint64_t)dr.xo.x < a.thr_c && ch.n >= 3) {                                   // a5
-            const uint32_t x = 1 + below(dr.xo.y, ch.n - 2);
+            const int x = (int)(1 + below(dr.xo.y, ch.n - 2));
 #pragma unroll
             for (int w = 0; w < WT; ++w) {
-                const uint32_t lo = 64u * w;
-                const uint64_t m = (x >= lo + 64) ? ~0ull : (x <= lo ? 0ull : ((1ull << (x - lo)) - 1));
+                // positions < x from A: per 32-bit half one BMSK of the clamped width
+                const uint32_t m0 = bmsk32((uint32_t)max(x - 64 * w, 0)), m1 = bmsk32((uint32_t)max(x - 64 * w - 32, 0));
+                const uint64_t m = ((uint64_t)m1 << 32) | m0;
                 A.w[w] = (A.w[w] & m) | (B.w[w] & ~m);
             }
         }
         if (tr) a.trace[(g - a.g_begin) * 16 + 13] = gtimer() + 0 * A.w[0];
         if ((uint64_t)dr.mu.x < a.thr_m)                                                   // a6 (R22)
             row_xor_bit(A, a.front_skip + below(dr.mu.y, ch.n - 1 - a.front_skip));
-        repair(a, A, gid, g);                                                              // a7
+        const uint32_t cuts = repair(a, A, gid, g);                                        // a7
         if (tr) a.trace[(g - a.g_begin) * 16 + 10] = gtimer() + 0 * A.w[0];
-        const double f = eval_regs(ch, sP, sO, A, nullptr, srow);                         // a2
+        const double f = eval_regs(ch, sP, sO, A, nullptr, srow, spo_s, cuts);             // a2
         if (tr) a.trace[(g - a.g_begin) * 16 + 11] = gtimer() + 0 * (uint64_t)__double_as_longlong(f);
         row_store(A, popn + (size_t)slot * W, W);
         fitn[slot] = f;
@@ -1398,14 +1617,23 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
         }
         __syncthreads();
         if (whole) {
-            cta_select_sorted(sm.skey, sm.sidx, S, K, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+            select_sorted(sm.skey, sm.sidx, S, K, sm, sm.ekey, sm.tsel);
             for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.tsel[r];
         } else {
-            const uint64_t want = (kWorstCap + K) / 2;  // aim between K and the capacity
+            // aim the collection at ~max(4K, 256) entries (up to 65,536 individuals: <= 512, so the
+            // warp select sorts it), between K and the capacity for larger islands
+            const uint64_t wide = (kWorstCap + K) / 2, narrow = 4ull * K > 256 ? 4ull * K : 256;
+            const uint64_t want = (N <= 65536u && narrow < wide) ? narrow : wide;
             uint64_t pts = (want * S) / N;             // sample points at or beyond the threshold
             pts = pts < 1 ? 1 : pts;
-            cta_select_sorted(sm.skey, sm.sidx, S, (uint32_t)pts, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx,
-                              sm.ekey, sm.tsel);
+            if (pts <= 8 && S == 16u * 128u && blockDim.x == 512) {
+                // the pts-th largest of the 2048 samples: every warp sorts its 128 and keeps its
+                // top 8 (the pts-th overall is among them), one warp sorts the 16 x 8
+                cta_top8_of_2048(sm.skey, sm.sidx, (uint32_t)pts, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+            } else {
+                cta_select_sorted(sm.skey, sm.sidx, S, (uint32_t)pts, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx,
+                                  sm.ekey, sm.tsel);
+            }
             if (threadIdx.x == 0) {
                 a.wthr[i] = sm.ekey[pts - 1];           // the smallest selected key: >= pts sample points reach it
                 a.wl_cnt[i] = 0;
@@ -1415,48 +1643,43 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
     if (whole) return;                                 // uniform across CTAs (N is)
     trace_sync(a, a.g_end - a.g_begin, 4);
     grid.sync();
-    // one pass over the islands (I N < 2^32, checked at create): each CTA counts its entries per
-    // island in shared memory, reserves one range per island with a single global atomic, then
-    // writes them (the count and write passes see the same entries)
+    // one pass over the islands (I N < 2^32, checked at create): an entry at or beyond its island's
+    // threshold takes a slot of the island's list with one warp-aggregated global atomic per warp,
+    // island and pass step (a few hundred entries qualify in all)
     const uint32_t total = I * N, gtid = blockIdx.x * blockDim.x + threadIdx.x, gstride = gridDim.x * blockDim.x;
-    uint32_t* lcnt = sm.hist;                          // [I] counts, [I] bases at +16
     uint64_t* lthr = (uint64_t*)(sm.hist + 32);        // [I] thresholds
-    if (threadIdx.x < 32) lcnt[threadIdx.x] = 0;
     if (threadIdx.x < I) lthr[threadIdx.x] = __ldcg(a.wthr + threadIdx.x);
     __syncthreads();
     // eight loads in flight per thread and pass (the pass is latency-bound, not bandwidth-bound)
     constexpr uint32_t U = 8;
-    auto scan = [&](bool write) {
-        for (uint32_t e0 = gtid; e0 < total; e0 += U * gstride) {
-            uint64_t wk[U];
+    const uint32_t lane = threadIdx.x & 31u;
+    for (uint32_t e0 = gtid - lane; e0 < total; e0 += U * gstride) {     // warp-uniform trip count
+        uint64_t wk[U];
 #pragma unroll
-            for (uint32_t u = 0; u < U; ++u) {
-                const uint32_t e = e0 + u * gstride;
-                const uint32_t i = e / N;
-                wk[u] = e < total ? ~fkey(__ldcg(a.fit[cur] + (size_t)i * a.Ns + (e - i * N))) : 0ull;
-            }
+        for (uint32_t u = 0; u < U; ++u) {
+            const uint32_t e = e0 + lane + u * gstride;
+            const uint32_t i = e / N;
+            wk[u] = e < total ? ~fkey(__ldcg(a.fit[cur] + (size_t)i * a.Ns + (e - i * N))) : 0ull;
+        }
 #pragma unroll
-            for (uint32_t u = 0; u < U; ++u) {
-                const uint32_t e = e0 + u * gstride;
-                const uint32_t i = e / N;
-                if (e < total && wk[u] >= lthr[i]) {
-                    const uint32_t p = atomicAdd(lcnt + i, 1u);
-                    if (write && lcnt[16 + i] + p < kWorstCap) {
-                        a.wl_key[(size_t)i * kWorstCap + lcnt[16 + i] + p] = wk[u];
-                        a.wl_idx[(size_t)i * kWorstCap + lcnt[16 + i] + p] = ~(e - i * N);
-                    }
+        for (uint32_t u = 0; u < U; ++u) {
+            const uint32_t e = e0 + lane + u * gstride;
+            const uint32_t i = e < total ? e / N : 0u;
+            const bool pass = e < total && wk[u] >= lthr[i];
+            if (__any_sync(0xFFFFFFFFu, pass)) {
+                const unsigned grp = __match_any_sync(0xFFFFFFFFu, pass ? i : 0xFFFFFFFFu);
+                const int lead = __ffs(grp) - 1;
+                uint32_t base = 0;
+                if (pass && (int)lane == lead) base = atomicAdd(a.wl_cnt + i, (uint32_t)__popc(grp));
+                base = __shfl_sync(0xFFFFFFFFu, base, lead);
+                const uint32_t p = base + __popc(grp & ((1u << lane) - 1u));
+                if (pass && p < kWorstCap) {
+                    a.wl_key[(size_t)i * kWorstCap + p] = wk[u];
+                    a.wl_idx[(size_t)i * kWorstCap + p] = ~(e - i * N);
                 }
             }
         }
-    };
-    scan(false);
-    __syncthreads();
-    if (threadIdx.x < I) {
-        lcnt[16 + threadIdx.x] = lcnt[threadIdx.x] ? atomicAdd(a.wl_cnt + threadIdx.x, lcnt[threadIdx.x]) : 0u;
-        lcnt[threadIdx.x] = 0;
     }
-    __syncthreads();
-    scan(true);
     trace_sync(a, a.g_end - a.g_begin, 5);
     grid.sync();
     trace_sync(a, a.g_end - a.g_begin, 6);
@@ -1473,7 +1696,7 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
                 sm.sidx[j] = __ldcg(a.wl_idx + (size_t)i * kWorstCap + j);
             }
             __syncthreads();
-            cta_select_sorted(sm.skey, sm.sidx, C, K, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+            select_sorted(sm.skey, sm.sidx, C, K, sm, sm.ekey, sm.tsel);
             for (uint32_t r = threadIdx.x; r < K; r += blockDim.x) a.wslot[(size_t)i * kMaxElite + r] = ~sm.tsel[r];
         }
     } else {
@@ -1508,7 +1731,7 @@ __device__ void import_migrants(const GaArgs& a, uint32_t i, uint32_t g, const S
     __syncthreads();
     const uint32_t take = a.K < nf ? a.K : nf;
     // the K best foreign migrants in order (f desc, source asc, rank asc) -> ekey/tsel[0..take)
-    cta_select_sorted(sm.skey, sm.sidx, nf, take, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, sm.ekey, sm.tsel);
+    select_sorted(sm.skey, sm.sidx, nf, take, sm, sm.ekey, sm.tsel);
     for (uint32_t j = threadIdx.x; j < take * W; j += blockDim.x) {
         const uint32_t r = j / W, w = j % W, e = sm.tsel[r];
         pop[(size_t)__ldcg(worst_slot + r) * W + w] = __ldcg(xblock(a, e / a.K) + (size_t)(e % a.K) * W + w);
@@ -1604,6 +1827,8 @@ __global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs 
     smem_layout(a, smem, &sm);
     cg::grid_group grid = cg::this_grid();
     stage_chain(sm.chain, a.ch, sm.mbar);
+    stage_bulk(sm.po, a.ch.po, a.ch.po_bytes, sm.mbar + 2);
+    const uint32_t spo_s = opaque32(smem_u32(sm.po));
     const uint32_t* sP = sm.chain;
     const uint32_t* sO = sm.chain + a.ch.p_words;
     const uint32_t W = a.ch.W, N = a.N, E = a.E, I = a.I, Ns = a.Ns, cpi = a.cpi, cpp = a.cpi_pad;
@@ -1628,7 +1853,7 @@ __global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs 
                 if (c >= N) continue;
                 Row<WT> r;
                 init_row(a, r, (a.island_base + i) * N + c);
-                const double f = eval_regs(a.ch, sP, sO, r, nullptr, sm.rows + threadIdx.x * (2 * W + 1));
+                const double f = eval_regs(a.ch, sP, sO, r, nullptr, sm.rows + threadIdx.x * (2 * W + 1), spo_s);
                 row_store(r, pop + (size_t)c * W, W);
                 fit[c] = f;
                 track_row(best, f, c, r, W);
@@ -1753,7 +1978,7 @@ __global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs 
                 a.trace[(g - a.g_begin) * 16 + 4] = gtimer();
             const size_t reg = ((size_t)i * cpi + my_local) * a.creg;    // this CTA's candidate region
             breed_children<WT>(a, i, g, my_local, a.pop[cur] + (size_t)i * N * W, a.fit[cur] + (size_t)i * Ns,
-                               a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO,
+                               a.pop[nxt] + (size_t)i * N * W, a.fit[nxt] + (size_t)i * Ns, sP, sO, spo_s,
                                a.tau + tau_par * I + i, sm.misc + 24, a.cand_key[Lb] + reg, a.cand_idx[Lb] + reg,
                                a.rc_cnt + Lb * I + i, a.rc_idx[Lb] + (size_t)i * Ns, snap, pre, have_pre,
                                have_fpre ? fpre : nullptr, sm.rows + threadIdx.x * (2 * W + 1));

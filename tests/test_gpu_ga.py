@@ -263,6 +263,18 @@ def test_c4_shaped_batched_islands(S):
              migration_interval=10, n_migrants=64)
 
 
+@pytest.mark.parametrize("N,K,I,M", [(8192, 32, 4, 3), (65536, 200, 3, 4), (3000, 16, 5, 2)])
+def test_sync_point_selection_paths(S, N, K, I, M):
+    """The sync point's selections take different paths by size (one-warp sort for
+    <= 512 entries, the radix select beyond; the collection threshold from a
+    two-level warp sort of the sample or the radix select): island sizes between the
+    whole-island sort and C4's 65,536, and a K whose collection exceeds one warp's
+    sort, all bit for bit against the oracle's serial islands."""
+    lat, ovh = wl.chain("vgg16")
+    run_both(S, lat, ovh, 3 * M + 1, 11, pop_size=N, n_elite=16, k_min=2, k_max=12, n_islands=I,
+             migration_interval=M, n_migrants=K)
+
+
 def test_comm_layout_checked_at_create(S):
     """A communicator of world 1 cannot host islands of another layout (advisor: the
     all-gathers would write past the buffers); the device must match too."""
