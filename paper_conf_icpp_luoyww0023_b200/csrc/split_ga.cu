@@ -124,24 +124,24 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, uint32_t 
     uint32_t endP = ch.T, OV = 0, v = 0, tb = spo_s;
     uint64_t S2 = 0;
     for (uint32_t j = 0; j < cuts; ++j) {
-        // refill (predicated): the next non-empty half when v is exhausted, chosen by a
-        // select tree over the bits of q (never a runtime register index)
-        const uint32_t q = bfind32(occ);
-        const bool need = (v == 0u);
-        uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
+        if (v == 0u) {
+            // refill: the next non-empty half, chosen by a select tree over the bits of q
+            // (never a runtime register index; a predicated refill was slower here: C2 7.2 ->
+            // 7.3 us per generation -- the tree's selects run on every cut)
+            const uint32_t q = bfind32(occ);
+            occ ^= 1u << q;
+            uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
 #pragma unroll
-        for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
-        uint32_t hv;
-        if constexpr (NH == 2) hv = t1[0];
-        else if constexpr (NH == 4) hv = (q & 2u) ? t1[1] : t1[0];
-        else {
-            const uint32_t a0 = (q & 2u) ? t1[1] : t1[0];
-            const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
-            hv = (q & 4u) ? a1 : a0;
+            for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
+            if constexpr (NH == 2) v = t1[0];
+            else if constexpr (NH == 4) v = (q & 2u) ? t1[1] : t1[0];
+            else {
+                const uint32_t a0 = (q & 2u) ? t1[1] : t1[0];
+                const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
+                v = (q & 4u) ? a1 : a0;
+            }
+            tb = spo_s + (q << 8);
         }
-        v = need ? hv : v;
-        occ = need ? (occ & bmsk32(q)) : occ;
-        tb = need ? spo_s + (q << 8) : tb;
         const uint32_t bt = bfind32(v);
         v &= bmsk32(bt);
         // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3):
@@ -873,14 +873,14 @@ __device__ __forceinline__ void warp_topm_lists(uint64_t (&k)[PER], uint32_t (&x
     }
 }
 
-// All 512 threads: the m largest (m <= 8) of 2048 entries in ranking order: every warp takes the top 8 of its
+// All threads (>= 512; 16 warps work): the m largest (m <= 8) of 2048 entries in ranking order: every warp takes the top 8 of its
 // 128 (lane-local sort of 4, then warp_topm_lists), one warp the top m of the 16 x 8.
 // tk/tx: 128-entry scratch.  The result goes to ok/ox[0..m).
 __device__ __forceinline__ void cta_top8_of_2048(const uint64_t* key, const uint32_t* idx, uint32_t m, uint64_t* tk,
                                                  uint32_t* tx, uint64_t* ok, uint32_t* ox)
 {
     const uint32_t w = threadIdx.x >> 5, lane = threadIdx.x & 31u;
-    {
+    if (w < 16u) {
         uint64_t k[4];
         uint32_t x[4];
 #pragma unroll
@@ -910,7 +910,7 @@ __device__ __forceinline__ void cta_top8_of_2048(const uint64_t* key, const uint
     __syncthreads();
 }
 
-// All 512 threads: sort n <= 512 entries of key/idx (shared memory) in the ranking order
+// All threads (>= 512; the first 512 work): sort n <= 512 entries of key/idx (shared memory) in the ranking order
 // and write the first m to ok/ox.  One entry per thread: each warp sorts its 32 by a
 // register bitonic network, then four merge levels (runs of 32 -> 512) place every entry
 // at its own position plus its rank in the partner run (binary search; the left run wins
@@ -920,6 +920,7 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
                             uint32_t* ox, uint64_t* bk, uint32_t* bx)
 {
     const uint32_t lane = threadIdx.x & 31u;
+    const bool act = threadIdx.x < 512u;        // whole warps: the shuffles below stay warp-uniform
     uint32_t t = threadIdx.x;
     uint64_t k[1];
     uint32_t x[1];
@@ -929,8 +930,10 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
     __syncthreads();                             // key/idx may be overwritten below
 #pragma unroll
     for (uint32_t L = 32; L < 512; L <<= 1) {
-        bk[t] = k[0];
-        bx[t] = x[0];
+        if (act) {
+            bk[t] = k[0];
+            bx[t] = x[0];
+        }
         __syncthreads();
         const uint32_t base = t & ~(2u * L - 1u), pos = t & (L - 1u);
         const bool left = (t & L) == 0u;
@@ -938,6 +941,7 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
         // left entries count the partner's strictly greater entries, right entries the
         // greater-or-equal ones (a prefix of the partner run): branch-free binary lifting
         uint32_t lo = 0;
+        if (act) {
 #pragma unroll
         for (uint32_t step = L >> 1; step > 0; step >>= 1) {
             const uint64_t km = bk[ob + lo + step - 1];
@@ -949,10 +953,11 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
             const uint32_t xm = bx[ob + lo];
             lo += (gt_nb(km, xm, k[0], x[0]) | (!left & !gt_nb(k[0], x[0], km, xm))) ? 1u : 0u;
         }
+        }
         __syncthreads();
         t = base + pos + lo;
     }
-    if (t < m) { ok[t] = k[0]; ox[t] = x[0]; }
+    if (act && t < m) { ok[t] = k[0]; ox[t] = x[0]; }
     __syncthreads();
 }
 
@@ -964,7 +969,7 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
 __device__ __noinline__ void select_sorted(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t k,
                                            const Smem& sm, uint64_t* ok, uint32_t* ox)
 {
-    if (n > 512u || blockDim.x != 512u) {
+    if (n > 512u || blockDim.x < 512u) {
         cta_select_sorted(key, idx, n, k, sm.hist, sm.sel, sm.misc + 4, sm.okey, sm.oidx, ok, ox);
         return;
     }
@@ -1225,6 +1230,7 @@ __device__ void leader_fast(const GaArgs& a, uint32_t i, uint32_t g, const Smem&
         const uint32_t cnt_off = Lc * I + i;
         const uint32_t rwin = Ns < kRecWin ? Ns : kRecWin;
         const uint32_t b = 16u + rwin * 4u + (E > 0 ? round16(E * 8u) + cpp * 4u : 0u);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // earlier generic writes to the targets
         mbar_arrive_expect_tx(sm.mbar + 1, b);
         bulk_g2s(sm.misc + 16, a.rc_cnt + (cnt_off & ~3u), 16u, sm.mbar + 1);
         bulk_g2s(sm.rcw, a.rc_idx[Lc] + (size_t)i * Ns, rwin * 4u, sm.mbar + 1);
@@ -1532,12 +1538,11 @@ __device__ __forceinline__ void breed_children(const GaArgs& a, uint32_t i, uint
         }
         if (tr) a.trace[(g - a.g_begin) * 16 + 9] = gtimer() + 0 * (A.w[0] ^ B.w[0]);
         if ((uint64_t)dr.xo.x < a.thr_c && ch.n >= 3) {                                   // a5
-            const int x = (int)(1 + below(dr.xo.y, ch.n - 2));
+            const uint32_t x = 1 + below(dr.xo.y, ch.n - 2);
 #pragma unroll
             for (int w = 0; w < WT; ++w) {
-                // positions < x from A: per 32-bit half one BMSK of the clamped width
-                const uint32_t m0 = bmsk32((uint32_t)max(x - 64 * w, 0)), m1 = bmsk32((uint32_t)max(x - 64 * w - 32, 0));
-                const uint64_t m = ((uint64_t)m1 << 32) | m0;
+                const uint32_t lo = 64u * w;
+                const uint64_t m = (x >= lo + 64) ? ~0ull : (x <= lo ? 0ull : ((1ull << (x - lo)) - 1));
                 A.w[w] = (A.w[w] & m) | (B.w[w] & ~m);
             }
         }
@@ -1626,7 +1631,7 @@ __device__ void select_worst(const GaArgs& a, uint32_t g, const Smem& sm, cg::gr
             const uint64_t want = (N <= 65536u && narrow < wide) ? narrow : wide;
             uint64_t pts = (want * S) / N;             // sample points at or beyond the threshold
             pts = pts < 1 ? 1 : pts;
-            if (pts <= 8 && S == 16u * 128u && blockDim.x == 512) {
+            if (pts <= 8 && S == 16u * 128u && blockDim.x >= 512) {
                 // the pts-th largest of the 2048 samples: every warp sorts its 128 and keeps its
                 // top 8 (the pts-th overall is among them), one warp sorts the 16 x 8
                 cta_top8_of_2048(sm.skey, sm.sidx, (uint32_t)pts, sm.okey, sm.oidx, sm.ekey, sm.tsel);

@@ -109,7 +109,7 @@ def test_zero_chain_ties(S):
     run_both(S, lat, ovh, 30, 5, pop_size=256, n_elite=4, k_min=2, k_max=12)
 
 
-@pytest.mark.parametrize("M,stall", [(3, 0), (0, 0), (4, 8)])
+@pytest.mark.parametrize("M,stall", [(3, 0), (0, 0), (4, 8), (2, 3)])
 def test_local_islands_with_migration(S, M, stall):
     lat, ovh = wl.chain("resnet50_175")
     run_both(S, lat, ovh, 13, 77, pop_size=128, n_elite=4, k_min=2, k_max=16, n_islands=4,
