@@ -106,6 +106,19 @@ struct EvalCfg {
 // half back (a rare, divergent store; an unconditional read-modify-write of
 // that half costs a 32-way bank conflict per warp: every lane's row has it in
 // the same bank).
+// min(x, 1) as one VIMNMX (the compiler otherwise emits ISETP + SEL for x != 0)
+__device__ __forceinline__ uint32_t nz1(uint32_t x)
+{
+    uint32_t r;
+    asm("min.u32 %0, %1, 1;" : "=r"(r) : "r"(x));
+    return r;
+}
+// occupancy nibble of four halves: bit i <=> half i non-empty (adds of disjoint bits: LEAs)
+__device__ __forceinline__ uint32_t nib4(const uint4& v)
+{
+    return nz1(v.x) + 2u * nz1(v.y) + 4u * nz1(v.z) + 8u * nz1(v.w);
+}
+
 __device__ __forceinline__ uint32_t comp4(const uint4& v, uint32_t i)
 {
     return i == 0 ? v.x : (i == 1 ? v.y : (i == 2 ? v.z : v.w));
@@ -127,7 +140,7 @@ __device__ __forceinline__ uint32_t row_occupancy(uint32_t* my, uint32_t lane, u
 #pragma unroll
         for (uint32_t j = 0; j < 8; ++j) {
             const uint4 v = my4[j ^ rsw];
-            occ |= (min(v.x, 1u) | (min(v.y, 1u) << 1) | (min(v.z, 1u) << 2) | (min(v.w, 1u) << 3)) << (4 * j);
+            occ += nib4(v) << (4 * j);
             if constexpr (EXACT) pc += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
             if (j == 7) ctop = v;                // for W = 16 the padding (qfull >= 30) lives in chunk 7
         }
