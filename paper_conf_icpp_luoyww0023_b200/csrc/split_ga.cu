@@ -106,30 +106,32 @@ __device__ __forceinline__ void row_toggle_rank(Row<WT>& row, const ChainDev& ch
 // row's 32-bit halves held in registers (the next non-empty half is chosen
 // from an occupancy mask with a select tree, never with a runtime index), so
 // the trip count is the child's cut count rather than a per-word maximum.
-// Same integer statistics and Eq. 2 tail as eval_walk (R3, R5').
+// Same integer statistics and Eq. 2 tail as eval_walk (R3, R5').  (The wide form's staged
+// {P[p+1], ovh[p]} pairs and the repair's cut count made C2 ~2.5 % slower here: 4.32 vs 4.22 ms
+// per 500-generation step; kept for wide rows only.)
 template <int WT>
-__device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, uint32_t spo_s, const Row<WT>& r, uint32_t cuts)
+__device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uint32_t* sP, const uint32_t* sO,
+                                                   const Row<WT>& r)
 {
     constexpr int NH = 2 * WT;
     uint32_t h[NH];
-    uint32_t occ = 0;
+    uint32_t occ = 0, cuts = 0;
 #pragma unroll
     for (int i = 0; i < NH; ++i) {
         const uint64_t wv = (i / 2 < (int)ch.W) ? (r.w[i / 2] & word_mask(ch, i / 2)) : 0ull;
         h[i] = (uint32_t)(wv >> (32 * (i & 1)));
         occ |= (h[i] != 0u ? 1u : 0u) << i;
+        cuts += __popc(h[i]);
     }
     const uint32_t k = cuts + 1;
     if (k < ch.k_min || k > ch.k_max) return -CUDART_INF;
-    uint32_t endP = ch.T, OV = 0, v = 0, tb = spo_s;
+    uint32_t endP = ch.T, OV = 0, v = 0, qb = 0;
     uint64_t S2 = 0;
     for (uint32_t j = 0; j < cuts; ++j) {
         if (v == 0u) {
-            // refill: the next non-empty half, chosen by a select tree over the bits of q
-            // (never a runtime register index; a predicated refill was slower here: C2 7.2 ->
-            // 7.3 us per generation -- the tree's selects run on every cut)
             const uint32_t q = bfind32(occ);
             occ ^= 1u << q;
+            // select tree over the halves by the bits of q
             uint32_t t1[NH / 2 > 0 ? NH / 2 : 1];
 #pragma unroll
             for (int i = 0; i < NH / 2; ++i) t1[i] = (q & 1u) ? h[2 * i + 1] : h[2 * i];
@@ -140,17 +142,17 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, uint32_t 
                 const uint32_t a1 = (q & 2u) ? t1[3] : t1[2];
                 v = (q & 4u) ? a1 : a0;
             }
-            tb = spo_s + (q << 8);
+            qb = q << 5;
         }
         const uint32_t bt = bfind32(v);
-        v &= bmsk32(bt);
-        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3):
-        // one LDS.64 of the staged pair {P[p+1], ovh[p]}
-        const uint2 e = lds64(tb + 8u * bt);
-        const uint32_t t = endP - e.x + e.y;
+        v ^= 1u << bt;
+        const uint32_t p = qb + bt;
+        // the block after cut p runs to the previous (higher) cut and pays ovh[p] (R3)
+        const uint32_t Pp = sP[p + 1], op = sO[p];
+        const uint32_t t = endP - Pp + op;
         S2 += (uint64_t)t * t;
-        OV += e.y;
-        endP = e.x;
+        OV += op;
+        endP = Pp;
     }
     S2 += (uint64_t)endP * endP;                 // first block: ops 0 .. c_1
     const uint64_t S1 = (uint64_t)ch.T + OV;
@@ -211,8 +213,13 @@ __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* 
                                             const Row<WT>& r, Stats* st, uint32_t* srow = nullptr,
                                             uint32_t spo_s = 0u, uint32_t cuts_known = ~0u)
 {
-    if constexpr (WT <= 16) {
-        if (!st && spo_s && (WT <= 4 || srow)) {
+    // (compile-time dispatch: a runtime test here keeps the generic walk below alive in the
+    // breeding loop, and its registers cost C2 ~2.4 %: 4.32 vs 4.22 ms per step)
+    if constexpr (WT <= 4) {
+        if (!st) return eval_regs_narrow<WT>(ch, sP, sO, r);
+    } else if constexpr (WT <= 16) {
+        if (!st) {
+            // wide rows: callers pass srow (this thread's row slot) and spo_s (the staged pairs)
             uint32_t c = cuts_known;
             if (c == ~0u) {
                 c = 0;
@@ -220,8 +227,7 @@ __device__ __forceinline__ double eval_regs(const ChainDev& ch, const uint32_t* 
                 for (int w = 0; w < WT; ++w)
                     if (w < (int)ch.W) c += __popcll(r.w[w] & word_mask(ch, w));
             }
-            if constexpr (WT <= 4) return eval_regs_narrow<WT>(ch, spo_s, r, c);
-            else return eval_wide<WT>(ch, spo_s, r, srow, c);
+            return eval_wide<WT>(ch, spo_s, r, srow, c);
         }
     }
     // same arithmetic as eval_walk, with the word loop unrolled over the register row
@@ -499,7 +505,7 @@ __host__ __device__ inline size_t smem_layout(const GaArgs& a, uint8_t* base, Sm
     uint8_t* p;
     p = take((size_t)(a.ch.p_words + a.ch.o_words) * 4); if (s) s->chain = (uint32_t*)p;
     p = take(32); if (s) s->mbar = (uint64_t*)p;
-    p = take(a.ch.po_bytes); if (s) s->po = (uint2*)p;
+    p = take((a.ch.W > 4 && a.ch.W <= 16) ? a.ch.po_bytes : 16); if (s) s->po = (uint2*)p;   // wide rows only
     p = take((size_t)a.I * 256 * 4); if (s) s->hist = (uint32_t*)p;
     p = take((size_t)a.I * sizeof(SelState)); if (s) s->sel = (SelState*)p;
     p = take(33 * (16 + 8 * (size_t)wt_of(a.ch.W))); if (s) s->scratch = (BestRef*)p;
@@ -1832,7 +1838,7 @@ __global__ void __launch_bounds__(kBlock, SPLIT_GA_MIN_BLOCKS) ga_kernel(GaArgs 
     smem_layout(a, smem, &sm);
     cg::grid_group grid = cg::this_grid();
     stage_chain(sm.chain, a.ch, sm.mbar);
-    stage_bulk(sm.po, a.ch.po, a.ch.po_bytes, sm.mbar + 2);
+    if (a.ch.W > 4 && a.ch.W <= 16) stage_bulk(sm.po, a.ch.po, a.ch.po_bytes, sm.mbar + 2);   // (uniform)
     const uint32_t spo_s = opaque32(smem_u32(sm.po));
     const uint32_t* sP = sm.chain;
     const uint32_t* sO = sm.chain + a.ch.p_words;
