@@ -972,7 +972,7 @@ __device__ void cta_sort512(const uint64_t* key, const uint32_t* idx, uint32_t n
 // the CTA has 512 threads, the radix select otherwise.  All threads of the CTA call it;
 // the inputs must be visible (a __syncthreads after they were written).  sm.okey/oidx
 // serve as scratch, as they do for the radix select.
-__device__ __noinline__ void select_sorted(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t k,
+__device__ __forceinline__ void select_sorted(const uint64_t* key, const uint32_t* idx, uint32_t n, uint32_t k,
                                            const Smem& sm, uint64_t* ok, uint32_t* ox)
 {
     if (n > 512u || blockDim.x < 512u) {
