@@ -49,13 +49,17 @@ __device__ __forceinline__ uint64_t word_mask(const ChainDev& ch, uint32_t w)
 {
     return (w + 1 == ch.W) ? ch.last_mask : ~0ull;
 }
+// Rows of the GA population never carry padding bits: init, mutation and repair place cuts only
+// at positions < n - 1, crossover and migration combine such rows; the register words past W
+// are zero (row_load).  So the GA counts and scans rows without masks or W bounds (the padding
+// masks stay where external bitsets are read: K1, split_eval.cu).
 template <int WT>
 __device__ __forceinline__ uint32_t row_popc(const Row<WT>& r, const ChainDev& ch)
 {
     uint32_t c = 0;
 #pragma unroll
     for (int i = 0; i < WT; ++i)
-        if (i < (int)ch.W) c += __popcll(r.w[i] & word_mask(ch, i));
+        c += __popcll(r.w[i]);
     return c;
 }
 
@@ -118,7 +122,7 @@ __device__ __forceinline__ double eval_regs_narrow(const ChainDev& ch, const uin
     uint32_t occ = 0, cuts = 0;
 #pragma unroll
     for (int i = 0; i < NH; ++i) {
-        const uint64_t wv = (i / 2 < (int)ch.W) ? (r.w[i / 2] & word_mask(ch, i / 2)) : 0ull;
+        const uint64_t wv = r.w[i / 2];                 // GA rows: no padding bits (row_popc)
         h[i] = (uint32_t)(wv >> (32 * (i & 1)));
         occ |= (h[i] != 0u ? 1u : 0u) << i;
         cuts += __popc(h[i]);
@@ -173,7 +177,7 @@ __device__ __forceinline__ double eval_wide(const ChainDev& ch, uint32_t spo_s, 
 #pragma unroll
     for (int i = 0; i < WT; ++i) {
         if (i < (int)ch.W) {
-            const uint64_t wv = r.w[i] & word_mask(ch, i);
+            const uint64_t wv = r.w[i];                  // GA rows: no padding bits (row_popc)
             const uint32_t lo = (uint32_t)wv, hi = (uint32_t)(wv >> 32);
             my[2 * i] = lo;
             my[2 * i + 1] = hi;
@@ -1408,7 +1412,7 @@ __device__ __forceinline__ uint32_t repair(const GaArgs& a, Row<WT>& row, uint32
         // a running prefix (no POPC) and clears the rr-th set bit of that word
         uint32_t cw[WT];
 #pragma unroll
-        for (int i = 0; i < WT; ++i) cw[i] = (i < (int)ch.W) ? (uint32_t)__popcll(row.w[i] & word_mask(ch, i)) : 0u;
+        for (int i = 0; i < WT; ++i) cw[i] = (uint32_t)__popcll(row.w[i]);   // no padding bits (row_popc)
         while (c > ch.k_max - 1) {
             uint32_t r = below(dr.next(), c);
             uint32_t wi = 0xFFFFFFFFu, rr = 0;
@@ -1417,7 +1421,7 @@ __device__ __forceinline__ uint32_t repair(const GaArgs& a, Row<WT>& row, uint32
             for (int i = 0; i < WT; ++i) {
                 const bool here = (wi == 0xFFFFFFFFu) && r < cw[i];
                 wi = here ? (uint32_t)i : wi;
-                mw = here ? (row.w[i] & word_mask(ch, i)) : mw;
+                mw = here ? row.w[i] : mw;
                 rr = here ? r : rr;
                 r -= (wi == 0xFFFFFFFFu) ? cw[i] : 0u;
             }
