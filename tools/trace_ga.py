@@ -47,6 +47,14 @@ def show(path):
             print(f"{name:32s} median {d[len(d) // 2] / 1e3:7.2f} us   p90 {d[int(len(d) * 0.9)] / 1e3:7.2f} us")
     per = sorted(int(rows[i + 1]["work_sync"]) - int(rows[i]["work_sync"]) for i in range(len(rows) - 1))
     print(f"{'generation (worker sync to sync)':32s} median {per[len(per) // 2] / 1e3:7.2f} us")
+    # generation by generation (the first ones of a run are the slow ones): sync-to-sync and the
+    # leader's phases, to see where the early generations spend their time
+    for i in range(min(len(rows) - 1, 24)):
+        r, q = rows[i], rows[i + 1]
+        ph = {name: (int(r[b]) - int(r[a])) / 1e3 for a, b, name in pairs if int(r[a]) and int(r[b])}
+        lead = " ".join(f"{n.split(': ')[-1]} {v:.1f}" for n, v in ph.items() if n.startswith("leader"))
+        work = " ".join(f"{n.split(' (')[0]} {v:.1f}" for n, v in ph.items() if not n.startswith("leader"))
+        print(f"gen {i:2d}: {(int(q['work_sync']) - int(r['work_sync'])) / 1e3:6.2f} us | {lead} | {work}")
 
 
 def arrivals(path):
