@@ -486,6 +486,110 @@ __global__ void __launch_bounds__(NWG * NG * 32, (48 / (NWG * NG)) > 0 ? 48 / (N
     }
 }
 
+// K1, grouped and double-buffered (tuning variant): like eval_grp_kernel, but each
+// group owns two chunk buffers -- the next chunk's TMA is in flight while the group
+// walks the current one (the single-buffered group waits for it after its
+// end-of-chunk barrier).  Twice the shared memory per group: half the warps per SM.
+template <int NWG, int NG>
+struct Grp2Cfg {
+    static constexpr uint32_t CHUNK = NWG * 32, H = 32;
+    static constexpr uint32_t kBoxes = (CHUNK + 255u) / 256u, kBoxRows = CHUNK / kBoxes;
+    static size_t smem(uint32_t po_bytes)
+    {
+        return (size_t)NG * 2 * CHUNK * 128 + po_bytes + 8 * (1 + 2 * NG + 1) + (size_t)NG * (CHUNK * 6 + 128) + 64;
+    }
+};
+
+template <int NWG, int NG>
+__global__ void __launch_bounds__(NWG * NG * 32, (24 / (NWG * NG)) > 0 ? 24 / (NWG * NG) : 1)
+    eval_grp2_kernel(ChainDev ch, const uint64_t* __restrict__ bits, uint64_t n_cand, double* __restrict__ out,
+                     const __grid_constant__ CUtensorMap tmap)
+{
+    using Cfg = Grp2Cfg<NWG, NG>;
+    constexpr uint32_t CHUNK = Cfg::CHUNK, H = Cfg::H, NTG = NWG * 32;
+    static_assert(CHUNK % 8 == 0 && Cfg::kBoxRows * Cfg::kBoxes == CHUNK, "swizzled chunk geometry");
+    extern __shared__ __align__(1024) uint8_t smem_grp2[];
+    const uint32_t tid = threadIdx.x, g = tid / NTG, gt = tid % NTG, lane = tid & 31u, gwarp = gt >> 5;
+    uint32_t* bufs = (uint32_t*)smem_grp2 + (size_t)g * 2 * CHUNK * H;     // this group's two chunk buffers
+    const uint2* spo = (const uint2*)(smem_grp2 + (size_t)NG * 2 * CHUNK * 128);
+    uint64_t* mbar = (uint64_t*)((const uint8_t*)spo + ch.po_bytes);       // [0] chain, [1 + 2g + b] buffers
+    uint8_t* gbase = (uint8_t*)(mbar + 1 + 2 * NG + 1) + (size_t)g * (CHUNK * 6 + 128);
+    uint32_t* s_occ = (uint32_t*)gbase;
+    uint32_t* s_hist = s_occ + CHUNK;
+    uint16_t* s_perm = (uint16_t*)(s_hist + 32);
+    if (tid == 0)
+        for (uint32_t q = 0; q < 2 * NG; ++q) mbar_init(mbar + 1 + q, 1);
+    if (gt < 32) s_hist[gt] = 0;
+    stage_bulk((void*)spo, ch.po, ch.po_bytes, mbar);
+    const uint32_t npos = ch.n - 1, qfull = npos >> 5;
+    const uint32_t lastm = (npos & 31u) ? ((1u << (npos & 31u)) - 1u) : 0u;
+    const uint32_t validocc = (qfull >= 32u) ? ~0u : ((1u << qfull) - 1u);
+    const uint32_t spo_s = opaque32(smem_u32(spo));
+    const uint64_t n_chunks = (n_cand + CHUNK - 1) / CHUNK;
+    const uint64_t stride = (uint64_t)gridDim.x * NG;
+    uint64_t c = (uint64_t)blockIdx.x * NG + g;
+    auto issue = [&](uint64_t cc, uint32_t b) {
+        if (gt == 0 && cc < n_chunks) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_expect_tx(mbar + 1 + 2 * g + b, CHUNK * 128u);
+#pragma unroll
+            for (uint32_t x = 0; x < Cfg::kBoxes; ++x) {
+                const int32_t y = (int32_t)(cc * CHUNK + x * Cfg::kBoxRows);
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                    ::"r"(smem_u32(bufs + b * CHUNK * H + x * Cfg::kBoxRows * H)), "l"(&tmap), "r"(0), "r"(y),
+                    "r"(smem_u32(mbar + 1 + 2 * g + b))
+                    : "memory");
+            }
+        }
+    };
+    issue(c, 0);
+    issue(c + stride, 1);
+    uint32_t ph = 0;                             // bit b: parity of buffer b's next phase
+    for (uint32_t b = 0; c < n_chunks; c += stride, b ^= 1u) {
+        uint32_t* buf = bufs + b * CHUNK * H;
+        const uint64_t row0 = c * CHUNK;
+        const uint32_t rows = (uint32_t)((n_cand - row0) < CHUNK ? (n_cand - row0) : CHUNK);
+        mbar_wait(mbar + 1 + 2 * g + b, (ph >> b) & 1u);
+        ph ^= 1u << b;
+        uint32_t key = 0, flags = 0x4000u;
+        if (gt < rows) {
+            uint32_t cuts;
+            const uint32_t occ = row_occupancy<16, false, true>(buf + gt * H, lane, validocc, qfull, lastm, cuts);
+            s_occ[gt] = occ;
+            const uint32_t ne = __popc(occ);
+            flags = (ne < ch.k_max && cuts < ch.k_max) ? 0u : 0x8000u;
+            key = flags ? 0u : min(cuts, 31u);
+        }
+        const uint32_t rank = atomicAdd(&s_hist[key], 1u);
+        named_bar(1 + g, NTG);
+        {
+            const uint32_t hv = s_hist[lane];
+            uint32_t inc = hv;
+#pragma unroll
+            for (uint32_t o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, inc, o);
+                if (lane >= o) inc += y;
+            }
+            const uint32_t start = __shfl_sync(0xFFFFFFFFu, inc - hv, key);
+            s_perm[start + rank] = (uint16_t)(gt | flags);
+        }
+        named_bar(1 + g, NTG);
+        if (gt < 32) s_hist[gt] = 0;
+        {
+            const uint32_t pe = s_perm[32u * gwarp + lane];
+            const uint32_t r = pe & 0x3FFFu;
+            if (!(pe & 0x4000u)) {
+                const double f = (pe & 0x8000u) ? -CUDART_INF
+                                                : walk_row<true>(ch, s_occ[r], smem_u32(buf + r * H), r, spo_s);
+                __stcs(out + row0 + r, f);
+            }
+        }
+        named_bar(1 + g, NTG);                    // buffer b, occupancy masks and order released
+        issue(c + 2 * stride, b);                 // buffer b takes the chunk after the one in flight
+    }
+}
+
 // ------------------------------------------------------------------------
 // Small kernels
 // ------------------------------------------------------------------------
@@ -537,6 +641,14 @@ static EvalVariant eval_grp_variant()
     EvalVariant v{(void*)eval_grp_kernel<NWG, NG>, 16u, (uint32_t)NWG, 1u, 1u, 1u};
     v.NG = NG;
     v.grp_smem = &GrpCfg<NWG, NG>::smem;
+    return v;
+}
+template <int NWG, int NG>
+static EvalVariant eval_grp2_variant()
+{
+    EvalVariant v{(void*)eval_grp2_kernel<NWG, NG>, 16u, (uint32_t)NWG, 1u, 1u, 1u};
+    v.NG = NG;
+    v.grp_smem = &Grp2Cfg<NWG, NG>::smem;
     return v;
 }
 
@@ -609,6 +721,10 @@ static EvalVariant eval_pick(uint32_t W)
         case 102: return eval_variant<16, 16, 1, 1, 0, true>();
         case 103: return eval_variant<16, 12, 1, 1, 0, true>();
         case 104: return eval_variant<16, 8, 2, 1, 0, true>();
+        case 500: return eval_grp2_variant<3, 4>();    // double-buffered groups: 2 CTAs x 4 x 3 warps per SM
+        case 501: return eval_grp2_variant<6, 2>();    // 2 CTAs x 2 x 6 warps
+        case 502: return eval_grp2_variant<4, 3>();    // 2 CTAs x 3 x 4 warps
+        case 503: return eval_grp2_variant<2, 6>();    // 2 CTAs x 6 x 2 warps
         case 400: return eval_grp_variant<6, 4>();     // 2 CTAs x 4 groups x 6 warps per SM
         case 401: return eval_grp_variant<5, 4>();
         case 402: return eval_grp_variant<8, 3>();
